@@ -1,0 +1,325 @@
+// eri_core.cuh -- per-class McMurchie-Davidson ERI machinery for sm_100a (FP64, DMMA).
+//
+// One warp evaluates one shell quartet (ab|cd) of class (la lb|lc ld) as the matrix-shaped
+// stages of PAPER.md Alg. 1 (L194-L213):
+//   a4 Boys F_m(T)              PAPER.md:L173-L177 (Taylor grid + downward recursion, reading R1)
+//   a5 R-tensor, Eq. 5          PAPER.md:L179-L180, warp-cooperative, level by level in SMEM
+//   a6 [p|q] = (-1)^{l_q}[p+q]  PAPER.md:L182-L184, gathered straight into DMMA B fragments through
+//                               an index table (the paper's SL->BL "transpose", L233-L249, without
+//                               materialising [p|q]); the sign is folded into E~_CD
+//   a7 GEMM1 [ab|q] += E~_AB [p|q]      PAPER.md:L186-L188 Eq. 7, mma.sync.m8n8k4.f64 (DMMA)
+//   a8 GEMM2 (ab|cd) += [ab|q] E~_CD^T  Eq. 7 / Eq. 11 (L251-L271), chained in registers: the
+//                               m8n8 accumulator of GEMM1 IS the A operand of GEMM2 (no SMEM trip)
+//   a9 digestion into FP64 J/K  (north_star; L296 FP64 accumulation)
+// The spherical transform, contraction coefficients and 1/p are folded into E~ (pairs.cu).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include "mako_internal.h"
+
+namespace mako {
+
+constexpr double TWO_PI_52 = 34.98683665524972497;  // 2 pi^{5/2}
+constexpr double PI_D = 3.14159265358979323846;
+
+MK_HD constexpr int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
+MK_HD constexpr int bla(int b) { return b >= 6 ? 3 : (b >= 3 ? 2 : (b >= 1 ? 1 : 0)); }
+MK_HD constexpr int blb(int b) { return b - bla(b) * (bla(b) + 1) / 2; }
+
+template <int LA_, int LB_, int LC_, int LD_>
+struct Cls {
+  static constexpr int LA = LA_, LB = LB_, LC = LC_, LD = LD_;
+  static constexpr int LAB = LA + LB, LCD = LC + LD, L = LAB + LCD;
+  static constexpr int NA = 2 * LA + 1, NB = 2 * LB + 1, NC = 2 * LC + 1, ND = 2 * LD + 1;
+  static constexpr int NAB = NA * NB, NCD = NC * ND;
+  static constexpr int NHAB = nH(LAB), NHCD = nH(LCD), NH = nH(L);
+  static constexpr int MT = (NAB + 7) / 8;    // m8 tiles over ab
+  static constexpr int NT1 = (NHCD + 7) / 8;  // GEMM1 n8 tiles over q
+  static constexpr int KS1 = (NHAB + 3) / 4;  // GEMM1 k4 steps over p
+  static constexpr int NT2 = (NCD + 7) / 8;   // GEMM2 n8 tiles over cd
+  // register budget for the accumulators (doubles per lane): MC m-tiles per chunk
+  static constexpr int REGB = 40;
+  static constexpr int MCMAX = clampi(REGB / (2 * (NT1 + NT2)), 1, MT);
+  static constexpr int NCHUNK = (MT + MCMAX - 1) / MCMAX;
+  static constexpr int MC = (MT + NCHUNK - 1) / NCHUNK;
+  // per-warp shared memory (doubles)
+  static constexpr int W_R = 2 * NH;    // ping-pong R levels
+  static constexpr int W_V = NAB * NCD; // (ab|cd) block
+  static constexpr int W_J = NAB;       // J_ab partial sums over the kets of a task
+  static constexpr int WARP_DBL = W_R + W_V + W_J;
+  // CTA tables
+  static constexpr int HTAB_BYTES = ((NHAB * NHCD * 2 + 15) / 16) * 16;
+  static constexpr int RTAB_BYTES = ((NH * 4 + 15) / 16) * 16;
+};
+
+template <int X, int Y>
+using ClsXY = Cls<bla(X), blb(X), bla(Y), blb(Y)>;
+
+// ---------------------------------------------------------------------------
+MK_HD inline void hdecode(int e, int& t, int& u, int& v) {
+  int k = 0;
+  while (nH(k) <= e) ++k;
+  int r = e - nH(k - 1);
+  int s = 0;
+  while ((s + 1) * (s + 2) / 2 <= r) ++s;
+  v = r - s * (s + 1) / 2;
+  u = s - v;
+  t = k - s;
+}
+
+// [pc][qc] -> Hermite index of p+q ; rtab[e] = packed recursion step for Hermite entry e
+template <class C>
+__device__ void init_tables(uint16_t* htab, uint32_t* rtab) {
+  for (int o = threadIdx.x; o < C::NHAB * C::NHCD; o += blockDim.x) {
+    int p = o / C::NHCD, q = o % C::NHCD, t1, u1, v1, t2, u2, v2;
+    hdecode(p, t1, u1, v1);
+    hdecode(q, t2, u2, v2);
+    htab[o] = (uint16_t)hidx(t1 + t2, u1 + u2, v1 + v2);
+  }
+  for (int e = threadIdx.x; e < C::NH; e += blockDim.x) {
+    uint32_t w = 0;
+    if (e > 0) {
+      int tt, uu, vv;
+      hdecode(e, tt, uu, vv);
+      int dir = tt > 0 ? 0 : (uu > 0 ? 1 : 2);
+      int n = dir == 0 ? tt : (dir == 1 ? uu : vv);
+      int s1 = dir == 0 ? hidx(tt - 1, uu, vv) : (dir == 1 ? hidx(tt, uu - 1, vv) : hidx(tt, uu, vv - 1));
+      int s2 = 0;
+      if (n >= 2) s2 = dir == 0 ? hidx(tt - 2, uu, vv) : (dir == 1 ? hidx(tt, uu - 2, vv) : hidx(tt, uu, vv - 2));
+      w = (uint32_t)s1 | ((uint32_t)s2 << 10) | ((uint32_t)dir << 20) | ((uint32_t)(n - 1) << 22);
+    }
+    rtab[e] = w;
+  }
+}
+
+// Boys F_m(T), m = 0..L: 7-term Taylor expansion of F_L about the nearest grid point, then the
+// downward recursion F_m = (2T F_{m+1} + e^{-T})/(2m+1); for T >= 40 the erf closed form of F_0
+// (erfc(sqrt 40) < 1e-18) and the upward recursion.
+template <int L>
+__device__ __forceinline__ void boys_eval(double T, const double* __restrict__ tab, double (&F)[L + 1]) {
+  if (T < BOYS_TMAX) {
+    const int k = __double2int_rn(T * (1.0 / BOYS_H));
+    const double x = k * BOYS_H - T;
+    const double* r = tab + k * BOYS_NM + L;
+    double f = __ldg(r + 6);
+    f = fma(f, x * (1.0 / 6.0), __ldg(r + 5));
+    f = fma(f, x * (1.0 / 5.0), __ldg(r + 4));
+    f = fma(f, x * 0.25, __ldg(r + 3));
+    f = fma(f, x * (1.0 / 3.0), __ldg(r + 2));
+    f = fma(f, x * 0.5, __ldg(r + 1));
+    f = fma(f, x, __ldg(r));
+    F[L] = f;
+    if constexpr (L > 0) {
+      const double e = exp(-T), t2 = 2.0 * T;
+#pragma unroll
+      for (int m = L - 1; m >= 0; --m) F[m] = fma(t2, F[m + 1], e) * (1.0 / (2 * m + 1));
+    }
+  } else {
+    const double it = 1.0 / T;
+    F[0] = 0.5 * sqrt(PI_D * it);
+    if constexpr (L > 0) {
+      const double e = exp(-T), h = 0.5 * it;
+#pragma unroll
+      for (int m = 0; m < L; ++m) F[m + 1] = fma((double)(2 * m + 1), F[m], -e) * h;
+    }
+  }
+}
+
+// R^{(0)}_{tuv}(rho, P-Q) for t+u+v <= L into buf[0..NH) (Eq. 4-5):
+//   R^{(n)}_{000} = (-2 rho)^n F_n(rho |PQ|^2) * 2 pi^{5/2} / sqrt(p+q)
+//   R^{(n)}_{t+1,u,v} = t R^{(n+1)}_{t-1,u,v} + X_PQ R^{(n+1)}_{t,u,v}   (and u, v alike)
+// Level n holds all entries with t+u+v <= L-n; lanes split each level; levels ping-pong.
+template <class C>
+__device__ __forceinline__ void compute_R(double p, double Px, double Py, double Pz, double q, double Qx, double Qy,
+                                          double Qz, double* __restrict__ buf, const uint32_t* __restrict__ rtab,
+                                          const double* __restrict__ btab, int lane) {
+  constexpr int L = C::L, NH = C::NH;
+  const double pq = p + q, rho = p * q / pq;
+  const double X = Px - Qx, Y = Py - Qy, Z = Pz - Qz;
+  const double T = rho * (X * X + Y * Y + Z * Z);
+  double F[L + 1];
+  boys_eval<L>(T, btab, F);
+  double s = TWO_PI_52 / sqrt(pq);
+  const double m2r = -2.0 * rho;
+#pragma unroll
+  for (int n = 0; n <= L; ++n) {
+    F[n] *= s;
+    s *= m2r;
+  }
+  if constexpr (L == 0) {
+    if (lane == 0) buf[0] = F[0];
+    __syncwarp();
+  } else {
+    if (lane == 0) buf[(L & 1) * NH] = F[L];
+    __syncwarp();
+#pragma unroll
+    for (int n = L - 1; n >= 0; --n) {
+      double* cur = buf + (n & 1) * NH;
+      const double* prv = buf + ((n + 1) & 1) * NH;
+      const int cnt = nH(L - n);
+      for (int e = lane; e < cnt; e += 32) {
+        double v;
+        if (e == 0) {
+          v = F[n];
+        } else {
+          const uint32_t w = rtab[e];
+          const int s1 = w & 1023, s2 = (w >> 10) & 1023, dir = (w >> 20) & 3, cf = (int)(w >> 22);
+          const double xd = dir == 0 ? X : (dir == 1 ? Y : Z);
+          v = xd * prv[s1];
+          if (cf) v = fma((double)cf, prv[s2], v);
+        }
+        cur[e] = v;
+      }
+      __syncwarp();
+    }
+  }
+}
+
+__device__ __forceinline__ void dmma884(double& c0, double& c1, double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+               : "+d"(c0), "+d"(c1)
+               : "d"(a), "d"(b));
+}
+
+// (ab|cd) block for bra pair P of `bra` and ket pair R of `ket` into V[ab][cd] (warp SMEM).
+// m8n8k4 f64 fragments (lane = 4g + t): A[g][t]; B[k=t][n=g]; C[g][2t+i].
+template <class C>
+__device__ void quartet_block(const PairView& bra, int P, const PairView& ket, int R, double* __restrict__ Rbuf,
+                              double* __restrict__ V, const uint16_t* __restrict__ htab,
+                              const uint32_t* __restrict__ rtab, const double* __restrict__ btab, int lane) {
+  const int g = lane >> 2, t = lane & 3;
+  const int b0 = __ldg(bra.poff + P), b1 = __ldg(bra.poff + P + 1);
+  const int k0 = __ldg(ket.poff + R), k1 = __ldg(ket.poff + R + 1);
+  for (int ch = 0; ch < C::NCHUNK; ++ch) {
+    double c2[C::MC][C::NT2][2];
+#pragma unroll
+    for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+      for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
+    for (int kl = k0; kl < k1; ++kl) {
+      const double q = __ldg(ket.pdat + 4 * kl), Qx = __ldg(ket.pdat + 4 * kl + 1), Qy = __ldg(ket.pdat + 4 * kl + 2),
+                   Qz = __ldg(ket.pdat + 4 * kl + 3);
+      double t1[C::MC][C::NT1][2];
+#pragma unroll
+      for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+        for (int nt = 0; nt < C::NT1; ++nt) t1[mc][nt][0] = t1[mc][nt][1] = 0.0;
+      for (int ij = b0; ij < b1; ++ij) {
+        const double p = __ldg(bra.pdat + 4 * ij), Px = __ldg(bra.pdat + 4 * ij + 1),
+                     Py = __ldg(bra.pdat + 4 * ij + 2), Pz = __ldg(bra.pdat + 4 * ij + 3);
+        compute_R<C>(p, Px, Py, Pz, q, Qx, Qy, Qz, Rbuf, rtab, btab, lane);
+        const double* __restrict__ E = bra.Ebra + (size_t)ij * (C::NAB * C::NHAB);
+#pragma unroll
+        for (int ks = 0; ks < C::KS1; ++ks) {
+          const int pc = 4 * ks + t;
+          double a[C::MC];
+#pragma unroll
+          for (int mc = 0; mc < C::MC; ++mc) {
+            const int row = 8 * (ch * C::MC + mc) + g;
+            a[mc] = (row < C::NAB && pc < C::NHAB) ? __ldg(E + row * C::NHAB + pc) : 0.0;
+          }
+#pragma unroll
+          for (int nt = 0; nt < C::NT1; ++nt) {
+            const int qc = 8 * nt + g;
+            const double b = (pc < C::NHAB && qc < C::NHCD) ? Rbuf[htab[pc * C::NHCD + qc]] : 0.0;
+#pragma unroll
+            for (int mc = 0; mc < C::MC; ++mc)
+              if (ch * C::MC + mc < C::MT) dmma884(t1[mc][nt][0], t1[mc][nt][1], a[mc], b);
+          }
+        }
+        __syncwarp();
+      }
+      // GEMM2: k-step (nt, e) takes q = 8 nt + 2 t + e from the GEMM1 accumulator of lane (g, t)
+      const double* __restrict__ Ek = ket.Eket + (size_t)kl * (C::NHCD * C::NCD);
+#pragma unroll
+      for (int nt = 0; nt < C::NT1; ++nt)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int qq = 8 * nt + 2 * t + e;
+#pragma unroll
+          for (int n2 = 0; n2 < C::NT2; ++n2) {
+            const int cd = 8 * n2 + g;
+            const double b = (qq < C::NHCD && cd < C::NCD) ? __ldg(Ek + qq * C::NCD + cd) : 0.0;
+#pragma unroll
+            for (int mc = 0; mc < C::MC; ++mc)
+              if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
+          }
+        }
+    }
+#pragma unroll
+    for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+      for (int n2 = 0; n2 < C::NT2; ++n2)
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int row = 8 * (ch * C::MC + mc) + g, col = 8 * n2 + 2 * t + i;
+          if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] = c2[mc][n2][i];
+        }
+  }
+  __syncwarp();
+}
+
+// Digestion of one canonical quartet (north_star J/K; FP64 accumulation).
+// With v' = deg * (ab|cd), deg = 1/2 per coincidence (a=b, c=d, ab=cd), the 8 permutations of a
+// canonical quartet reduce for symmetric D to the 6 forward updates below; the transposed halves
+// are restored by J = Jacc + Jacc^T, K = Kacc + Kacc^T at the end of the build.
+template <class C>
+__device__ void digest(const double* __restrict__ V, double deg, int oa, int ob, int oc, int od,
+                       const double* __restrict__ D, int nbf, double* __restrict__ J, double* __restrict__ K,
+                       double* __restrict__ jab, int lane) {
+  // J_ab (accumulated in SMEM across the kets of the task)
+  for (int ab = lane; ab < C::NAB; ab += 32) {
+    double s = 0.0;
+#pragma unroll 4
+    for (int cd = 0; cd < C::NCD; ++cd)
+      s = fma(V[ab * C::NCD + cd], __ldg(D + (size_t)(oc + cd / C::ND) * nbf + od + cd % C::ND), s);
+    jab[ab] = fma(2.0 * deg, s, jab[ab]);
+  }
+  // J_cd
+  for (int cd = lane; cd < C::NCD; cd += 32) {
+    double s = 0.0;
+#pragma unroll 4
+    for (int ab = 0; ab < C::NAB; ++ab)
+      s = fma(V[ab * C::NCD + cd], __ldg(D + (size_t)(oa + ab / C::NB) * nbf + ob + ab % C::NB), s);
+    atomicAdd(J + (size_t)(oc + cd / C::ND) * nbf + od + cd % C::ND, 2.0 * deg * s);
+  }
+  // K_ac += v D_bd
+  for (int x = lane; x < C::NA * C::NC; x += 32) {
+    const int i = x / C::NC, k = x % C::NC;
+    double s = 0.0;
+    for (int j = 0; j < C::NB; ++j)
+      for (int l = 0; l < C::ND; ++l)
+        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(ob + j) * nbf + od + l), s);
+    atomicAdd(K + (size_t)(oa + i) * nbf + oc + k, deg * s);
+  }
+  // K_ad += v D_bc
+  for (int x = lane; x < C::NA * C::ND; x += 32) {
+    const int i = x / C::ND, l = x % C::ND;
+    double s = 0.0;
+    for (int j = 0; j < C::NB; ++j)
+      for (int k = 0; k < C::NC; ++k)
+        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(ob + j) * nbf + oc + k), s);
+    atomicAdd(K + (size_t)(oa + i) * nbf + od + l, deg * s);
+  }
+  // K_bc += v D_ad
+  for (int x = lane; x < C::NB * C::NC; x += 32) {
+    const int j = x / C::NC, k = x % C::NC;
+    double s = 0.0;
+    for (int i = 0; i < C::NA; ++i)
+      for (int l = 0; l < C::ND; ++l)
+        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(oa + i) * nbf + od + l), s);
+    atomicAdd(K + (size_t)(ob + j) * nbf + oc + k, deg * s);
+  }
+  // K_bd += v D_ac
+  for (int x = lane; x < C::NB * C::ND; x += 32) {
+    const int j = x / C::ND, l = x % C::ND;
+    double s = 0.0;
+    for (int i = 0; i < C::NA; ++i)
+      for (int k = 0; k < C::NC; ++k)
+        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(oa + i) * nbf + oc + k), s);
+    atomicAdd(K + (size_t)(ob + j) * nbf + od + l, deg * s);
+  }
+}
+
+}  // namespace mako

@@ -1,0 +1,194 @@
+// eri_kernels.cuh -- per-class kernels (J/K build, batch store, Schwarz diagonal) and launchers.
+// Included with MAKO_DEFINE_KERNELS by the eri_cls_*.cu translation units (one per bra bucket),
+// without it by the dispatcher (declarations only).
+#pragma once
+
+#include "mako_state.h"
+
+namespace mako {
+
+constexpr int CTA_THREADS = 128;
+constexpr int CTA_WARPS = CTA_THREADS / 32;
+
+template <int X, int Y>
+mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch);
+template <int X, int Y>
+mako_status launch_batch_xy(const BatchArgs& a, void* stream);
+template <int X, int Y>
+int jk_blocks_per_sm();
+
+}  // namespace mako
+
+#ifdef MAKO_DEFINE_KERNELS
+#include "eri_core.cuh"
+
+namespace mako {
+
+template <class C>
+__host__ __device__ constexpr size_t cta_smem_bytes() {
+  return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)CTA_WARPS * C::WARP_DBL;
+}
+
+// Persistent J/K kernel: each warp pulls tasks (bra pair, <= KT consecutive kets) from a global counter.
+template <int X, int Y>
+__global__ void __launch_bounds__(CTA_THREADS) jk_kernel(JKArgs a) {
+  using C = ClsXY<X, Y>;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  uint16_t* htab = reinterpret_cast<uint16_t*>(smem_raw);
+  uint32_t* rtab = reinterpret_cast<uint32_t*>(smem_raw + C::HTAB_BYTES);
+  double* wbase = reinterpret_cast<double*>(smem_raw + C::HTAB_BYTES + C::RTAB_BYTES);
+  init_tables<C>(htab, rtab);
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  double* Rbuf = wbase + (size_t)warp * C::WARP_DBL;
+  double* V = Rbuf + C::W_R;
+  double* jab = V + C::W_V;
+  for (;;) {
+    unsigned long long tk = 0;
+    if (lane == 0) tk = atomicAdd(a.counter, 1ull);
+    tk = __shfl_sync(0xffffffffu, tk, 0);
+    const long long task = a.task_begin + (long long)tk;
+    if (task >= a.task_end) break;
+    // bra = largest P with task_off[P] <= task
+    int lo = 0, hi = a.nbra - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (__ldg(a.task_off + mid) <= task) lo = mid; else hi = mid - 1;
+    }
+    const int P = lo;
+    const int r0 = (int)(task - __ldg(a.task_off + P)) * a.KT;
+    const int r1 = min(r0 + a.KT, __ldg(a.nket + P));
+    const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
+    const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
+    const double QP = __ldg(a.bra.Q + P);
+    for (int i = lane; i < C::NAB; i += 32) jab[i] = 0.0;
+    __syncwarp();
+    for (int R = r0; R < r1; ++R) {
+      if (QP * __ldg(a.ket.Q + R) < a.thresh) continue;
+      const int sc = __ldg(a.ket.shA + R), sd = __ldg(a.ket.shB + R);
+      quartet_block<C>(a.bra, P, a.ket, R, Rbuf, V, htab, rtab, a.boys, lane);
+      double deg = 1.0;
+      if (sa == sb) deg *= 0.5;
+      if (sc == sd) deg *= 0.5;
+      if (a.same_bucket && P == R) deg *= 0.5;
+      digest<C>(V, deg, oa, ob, __ldg(a.ao + sc), __ldg(a.ao + sd), a.D, a.nbf, a.J, a.K, jab, lane);
+      __syncwarp();
+    }
+    for (int ab = lane; ab < C::NAB; ab += 32)
+      atomicAdd(a.J + (size_t)(oa + ab / C::NB) * a.nbf + ob + ab % C::NB, jab[ab]);
+    __syncwarp();
+  }
+}
+
+// Batch kernel: one warp per listed quartet; store (eri_batch) or Schwarz-diagonal epilogue.
+template <int X, int Y>
+__global__ void __launch_bounds__(CTA_THREADS) batch_kernel(BatchArgs a) {
+  using C = ClsXY<X, Y>;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  uint16_t* htab = reinterpret_cast<uint16_t*>(smem_raw);
+  uint32_t* rtab = reinterpret_cast<uint32_t*>(smem_raw + C::HTAB_BYTES);
+  double* wbase = reinterpret_cast<double*>(smem_raw + C::HTAB_BYTES + C::RTAB_BYTES);
+  init_tables<C>(htab, rtab);
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  double* Rbuf = wbase + (size_t)warp * C::WARP_DBL;
+  double* V = Rbuf + C::W_R;
+  for (int qi = blockIdx.x * CTA_WARPS + warp; qi < a.nq; qi += gridDim.x * CTA_WARPS) {
+    const int P = a.qbra[qi], R = a.qket[qi];
+    quartet_block<C>(a.bra, P, a.ket, R, Rbuf, V, htab, rtab, a.boys, lane);
+    if (a.diag) {
+      double m = 0.0;
+      for (int ab = lane; ab < C::NAB; ab += 32) m = fmax(m, fabs(V[ab * C::NCD + ab]));
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+      if (lane == 0) a.out[a.qout[qi]] = sqrt(m);
+    } else {
+      // canonical V[A][B][C][D] -> user order [a][b][c][d] (undo the swaps)
+      const int fl = a.qflag[qi];
+      const bool sab = fl & 1, scd = fl & 2, sbk = fl & 4;
+      int n[4] = {C::NA, C::NB, C::NC, C::ND};
+      // sizes in user order
+      int nu[4];
+      {
+        // user positions of the canonical shells A, B, C, D
+        int posA = sbk ? (scd ? 3 : 2) : (sab ? 1 : 0);
+        int posB = sbk ? (scd ? 2 : 3) : (sab ? 0 : 1);
+        int posC = sbk ? (sab ? 1 : 0) : (scd ? 3 : 2);
+        int posD = sbk ? (sab ? 0 : 1) : (scd ? 2 : 3);
+        nu[posA] = n[0]; nu[posB] = n[1]; nu[posC] = n[2]; nu[posD] = n[3];
+        const size_t base = (size_t)a.qout[qi];
+        for (int e = lane; e < C::NAB * C::NCD; e += 32) {
+          int idx[4];
+          int ab = e / C::NCD, cd = e % C::NCD;
+          idx[posA] = ab / C::NB; idx[posB] = ab % C::NB; idx[posC] = cd / C::ND; idx[posD] = cd % C::ND;
+          a.out[base + (((size_t)idx[0] * nu[1] + idx[1]) * nu[2] + idx[2]) * nu[3] + idx[3]] = V[e];
+        }
+      }
+    }
+    __syncwarp();
+  }
+}
+
+template <int X, int Y>
+static mako_status set_smem_attr(const void* fn, size_t smem) {
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("cudaFuncSetAttribute: ") + cudaGetErrorString(e));
+  return MAKO_OK;
+}
+
+template <int X, int Y>
+int jk_blocks_per_sm() {
+  using C = ClsXY<X, Y>;
+  constexpr size_t smem = cta_smem_bytes<C>();
+  static int cached = -1;
+  if (cached < 0) {
+    if (set_smem_attr<X, Y>((const void*)jk_kernel<X, Y>, smem)) return 1;
+    int nb = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel<X, Y>, CTA_THREADS, smem);
+    cached = nb < 1 ? 1 : nb;
+  }
+  return cached;
+}
+
+template <int X, int Y>
+mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
+  using C = ClsXY<X, Y>;
+  constexpr size_t smem = cta_smem_bytes<C>();
+  const long long ntask = a.task_end - a.task_begin;
+  if (ntask <= 0) return MAKO_OK;
+  int dev = 0, nsm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  const int bps = jk_blocks_per_sm<X, Y>();
+  long long want = (ntask + CTA_WARPS - 1) / CTA_WARPS;
+  long long cap = (long long)nsm * bps;
+  const int grid = (int)(want < cap ? want : cap);
+  jk_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("jk_kernel launch: ") + cudaGetErrorString(e));
+  if (nlaunch) ++*nlaunch;
+  return MAKO_OK;
+}
+
+template <int X, int Y>
+mako_status launch_batch_xy(const BatchArgs& a, void* stream) {
+  using C = ClsXY<X, Y>;
+  constexpr size_t smem = cta_smem_bytes<C>();
+  if (a.nq <= 0) return MAKO_OK;
+  mako_status st = set_smem_attr<X, Y>((const void*)batch_kernel<X, Y>, smem);
+  if (st) return st;
+  int grid = (a.nq + CTA_WARPS - 1) / CTA_WARPS;
+  if (grid > 148 * 64) grid = 148 * 64;
+  batch_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("batch_kernel launch: ") + cudaGetErrorString(e));
+  return MAKO_OK;
+}
+
+}  // namespace mako
+
+#define MAKO_INSTANTIATE(X, Y)                                                                   \
+  template mako_status mako::launch_jk_xy<X, Y>(const mako::JKArgs&, void*, int*);               \
+  template mako_status mako::launch_batch_xy<X, Y>(const mako::BatchArgs&, void*);               \
+  template int mako::jk_blocks_per_sm<X, Y>();
+#endif

@@ -1,0 +1,359 @@
+// jk.cu -- mako_build_jk (the hot path), per-threshold quartet plans, sharding, eri_batch, boys.
+//
+// Plan: classes (X|Y) over pair buckets X >= Y (55 for l <= 3).  Within a
+// bucket pairs are sorted by Q descending, so for bra P the kets with Q_P Q_R >= thresh are a
+// PREFIX of bucket Y (clipped to R <= P when X == Y: canonical ab >= cd).  A task is (P, <= KT
+// consecutive kets of that prefix); tasks of a class are numbered by a prefix sum over P.
+// Sharding: shard s of n takes tasks [T s/n, T (s+1)/n) of every class.
+#include <algorithm>
+#include <cmath>
+
+#include "eri_kernels.cuh"
+#include "eri_core.cuh"
+
+namespace mako {
+
+// ----- dispatch over the 55 classes ----------------------------------------
+#define MAKO_CLASS_LIST(F)                                                                                      \
+  F(0, 0) F(1, 0) F(1, 1) F(2, 0) F(2, 1) F(2, 2) F(3, 0) F(3, 1) F(3, 2) F(3, 3) F(4, 0) F(4, 1) F(4, 2)      \
+  F(4, 3) F(4, 4) F(5, 0) F(5, 1) F(5, 2) F(5, 3) F(5, 4) F(5, 5) F(6, 0) F(6, 1) F(6, 2) F(6, 3) F(6, 4)       \
+  F(6, 5) F(6, 6) F(7, 0) F(7, 1) F(7, 2) F(7, 3) F(7, 4) F(7, 5) F(7, 6) F(7, 7) F(8, 0) F(8, 1) F(8, 2)       \
+  F(8, 3) F(8, 4) F(8, 5) F(8, 6) F(8, 7) F(8, 8) F(9, 0) F(9, 1) F(9, 2) F(9, 3) F(9, 4) F(9, 5) F(9, 6)       \
+  F(9, 7) F(9, 8) F(9, 9)
+
+mako_status launch_jk_class(int X, int Y, const JKArgs& a, void* stream, int* nl) {
+#define MAKO_JK_CASE(x, y) \
+  if (X == x && Y == y) return launch_jk_xy<x, y>(a, stream, nl);
+  MAKO_CLASS_LIST(MAKO_JK_CASE)
+#undef MAKO_JK_CASE
+  return fail(MAKO_ERR_UNSUPPORTED, "unknown class");
+}
+
+mako_status launch_batch_class(int X, int Y, const BatchArgs& a, void* stream) {
+#define MAKO_B_CASE(x, y) \
+  if (X == x && Y == y) return launch_batch_xy<x, y>(a, stream);
+  MAKO_CLASS_LIST(MAKO_B_CASE)
+#undef MAKO_B_CASE
+  return fail(MAKO_ERR_UNSUPPORTED, "unknown class");
+}
+
+static mako_status cuda_check(cudaError_t e, const char* what) {
+  if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+  return MAKO_OK;
+}
+
+template <class T>
+static mako_status upload(DevBuf& d, const std::vector<T>& h) {
+  mako_status st = d.alloc(h.size() * sizeof(T));
+  if (st) return st;
+  if (!h.empty()) return cuda_check(cudaMemcpy(d.p, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice), "upload");
+  return MAKO_OK;
+}
+
+// number of kets R of bucket Y (Q-sorted desc) with QP * Q[R] >= thresh
+static int prefix_count(const std::vector<double>& QY, double QP, double thresh) {
+  int lo = 0, hi = (int)QY.size();
+  while (lo < hi) {
+    int mid = (lo + hi) / 2;
+    if (QP * QY[mid] >= thresh) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+static mako_status ensure_plan(mako_pairs P, double thresh) {
+  if (P->plan.thresh == thresh && !P->plan.cls.empty()) return MAKO_OK;
+  Plan& pl = P->plan;
+  pl.cls.clear();
+  pl.cls.resize(NBUCKET * (NBUCKET + 1) / 2);
+  pl.KT = 16;
+  for (int X = 0; X < NBUCKET; ++X)
+    for (int Y = 0; Y <= X; ++Y) {
+      ClassPlan& c = pl.cls[class_index(X, Y)];
+      c.X = X;
+      c.Y = Y;
+      const PairBucket& bx = P->set.b[X];
+      const PairBucket& by = P->set.b[Y];
+      const int nbra = bx.n();
+      c.nket.assign(nbra, 0);
+      c.task_off.assign(nbra + 1, 0);
+      for (int p = 0; p < nbra; ++p) {
+        int nk = by.n() ? prefix_count(by.Q, bx.Q[p], thresh) : 0;
+        if (X == Y) nk = std::min(nk, p + 1);
+        c.nket[p] = nk;
+        c.nquartet += nk;
+        c.task_off[p + 1] = c.task_off[p] + (nk + pl.KT - 1) / pl.KT;
+      }
+      c.ntask = c.task_off[nbra];
+      mako_status st;
+      if (c.ntask > 0 && ((st = upload(c.d_nket, c.nket)) || (st = upload(c.d_task_off, c.task_off)))) return st;
+    }
+  pl.thresh = thresh;
+  return MAKO_OK;
+}
+
+// J = Jacc + Jacc^T, K = Kacc + Kacc^T (in place)
+__global__ void symmetrize_kernel(double* __restrict__ J, double* __restrict__ K, int n) {
+  const long long total = (long long)n * n;
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < total; x += (long long)gridDim.x * blockDim.x) {
+    const int i = (int)(x / n), j = (int)(x % n);
+    if (j > i) continue;
+    const size_t a = (size_t)i * n + j, b = (size_t)j * n + i;
+    const double sj = J[a] + J[b], sk = K[a] + K[b];
+    J[a] = sj; J[b] = sj;
+    K[a] = sk; K[b] = sk;
+  }
+}
+
+__global__ void boys_kernel(int n, const double* __restrict__ T, double* __restrict__ out, const double* __restrict__ tab,
+                            int mmax) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  double F[4 * LMAX + 1];
+  switch (mmax) {
+#define BCASE(m)                                                                   \
+  case m: {                                                                        \
+    double G[m + 1];                                                               \
+    boys_eval<m>(T[i], tab, G);                                                    \
+    for (int k = 0; k <= m; ++k) F[k] = G[k];                                      \
+    break;                                                                         \
+  }
+    BCASE(0) BCASE(1) BCASE(2) BCASE(3) BCASE(4) BCASE(5) BCASE(6) BCASE(7) BCASE(8) BCASE(9) BCASE(10) BCASE(11)
+    BCASE(12)
+#undef BCASE
+  }
+  for (int k = 0; k <= mmax; ++k) out[(size_t)i * (mmax + 1) + k] = F[k];
+}
+
+}  // namespace mako
+
+using namespace mako;
+
+static mako_status check_pairs(mako_pairs p) {
+  if (!p || !p->basis) return fail(MAKO_ERR_INVALID, "NULL pairs");
+  int dev = -1;
+  cudaGetDevice(&dev);
+  if (dev != p->basis->device) return fail(MAKO_ERR_STATE, "pairs belong to another CUDA device");
+  return MAKO_OK;
+}
+
+extern "C" mako_status mako_pairs_stats(mako_pairs p, double thresh, long long* n_pairs, long long* n_prim_pairs,
+                                        long long* n_quartets) {
+  try {
+    mako_status st;
+    if ((st = check_pairs(p))) return st;
+    if (!(thresh >= 0)) return fail(MAKO_ERR_INVALID, "thresh < 0");
+    thresh = std::max(thresh, p->tau);
+    if ((st = ensure_plan(p, thresh))) return st;
+    long long np = 0, npp = 0, nq = 0;
+    for (int b = 0; b < NBUCKET; ++b) {
+      np += p->set.b[b].n();
+      npp += p->set.b[b].poff.back();
+    }
+    for (auto& c : p->plan.cls) nq += c.nquartet;
+    if (n_pairs) *n_pairs = np;
+    if (n_prim_pairs) *n_prim_pairs = npp;
+    if (n_quartets) *n_quartets = nq;
+    return MAKO_OK;
+  } catch (const std::exception& e) {
+    return fail(MAKO_ERR_OOM, e.what());
+  }
+}
+
+extern "C" mako_status mako_pairs_flops(mako_pairs p, double thresh, int shard, int nshards, double* gemm_flops,
+                                        long long* n_quartets, long long* n_prim_quartets) {
+  try {
+    mako_status st;
+    if ((st = check_pairs(p))) return st;
+    if (!(thresh >= 0) || nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "bad args");
+    thresh = std::max(thresh, p->tau);
+    if ((st = ensure_plan(p, thresh))) return st;
+    double fl = 0;
+    long long nq = 0, npq = 0;
+    const int KT = p->plan.KT;
+    for (auto& c : p->plan.cls) {
+      const PairBucket& bx = p->set.b[c.X];
+      const PairBucket& by = p->set.b[c.Y];
+      const int la = bx.la, lb = bx.lb, lc = by.la, ld = by.lb;
+      const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
+      const double hab = nH(la + lb), hcd = nH(lc + ld);
+      const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
+      // ket prefix of bra P restricted to this shard's tasks; by.poff is the prefix sum of K_CD
+      for (int P = 0; P < (int)c.nket.size(); ++P) {
+        const long long a0 = c.task_off[P], a1 = c.task_off[P + 1];
+        if (a1 <= t0 || a0 >= t1) continue;
+        const long long KAB = bx.poff[P + 1] - bx.poff[P];
+        const int r0 = (int)(std::max(a0, t0) - a0) * KT;
+        const int r1 = std::min((int)(std::min(a1, t1) - a0) * KT, c.nket[P]);
+        if (r1 <= r0) continue;
+        const long long sumK = by.poff[r1] - by.poff[r0];
+        fl += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)sumK * 2.0 * nab * hcd * ncd;
+        nq += r1 - r0;
+        npq += KAB * sumK;
+      }
+    }
+    if (gemm_flops) *gemm_flops = fl;
+    if (n_quartets) *n_quartets = nq;
+    if (n_prim_quartets) *n_prim_quartets = npq;
+    return MAKO_OK;
+  } catch (const std::exception& e) {
+    return fail(MAKO_ERR_OOM, e.what());
+  }
+}
+
+extern "C" mako_status mako_build_jk_launches(mako_pairs p, double thresh, int shard, int nshards, int* n) {
+  mako_status st;
+  if ((st = check_pairs(p))) return st;
+  if (!n || !(thresh >= 0) || nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "bad args");
+  thresh = std::max(thresh, p->tau);
+  if ((st = ensure_plan(p, thresh))) return st;
+  int cnt = 1;  // symmetrize
+  for (auto& c : p->plan.cls) {
+    const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
+    if (t1 > t0) ++cnt;
+  }
+  *n = cnt;
+  return MAKO_OK;
+}
+
+extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thresh, double* J, double* K, int shard,
+                                     int nshards, void* cuda_stream) {
+  try {
+    mako_status st;
+    if ((st = check_pairs(p))) return st;
+    if (!D || !J || !K) return fail(MAKO_ERR_INVALID, "NULL matrix");
+    if (D == J || D == K || J == K) return fail(MAKO_ERR_INVALID, "D, J, K must not alias");
+    if (!(thresh >= 0) || !std::isfinite(thresh)) return fail(MAKO_ERR_INVALID, "thresh must be finite and >= 0");
+    if (nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "shard out of range");
+    thresh = std::max(thresh, p->tau);
+    if ((st = ensure_plan(p, thresh))) return st;
+    const mako_basis_s* B = p->basis;
+    const int n = B->nbf;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    if ((st = cuda_check(cudaMemsetAsync(J, 0, sizeof(double) * n * n, s), "memset J")) ||
+        (st = cuda_check(cudaMemsetAsync(K, 0, sizeof(double) * n * n, s), "memset K")) ||
+        (st = cuda_check(cudaMemsetAsync(p->d_counters.p, 0, sizeof(unsigned long long) * 64, s), "memset ctr")))
+      return st;
+    int nl = 0;
+    for (auto& c : p->plan.cls) {
+      JKArgs a{};
+      a.task_begin = c.ntask * shard / nshards;
+      a.task_end = c.ntask * (shard + 1) / nshards;
+      if (a.task_end <= a.task_begin) continue;
+      a.bra = p->set.b[c.X].view();
+      a.ket = p->set.b[c.Y].view();
+      a.same_bucket = c.X == c.Y;
+      a.task_off = c.d_task_off.as<long long>();
+      a.nket = c.d_nket.as<int>();
+      a.nbra = (int)c.nket.size();
+      a.KT = p->plan.KT;
+      a.counter = p->d_counters.as<unsigned long long>() + class_index(c.X, c.Y);
+      a.D = D;
+      a.J = J;
+      a.K = K;
+      a.nbf = n;
+      a.ao = B->d_ao.as<int>();
+      a.thresh = thresh;
+      a.boys = B->d_boys.as<double>();
+      if ((st = launch_jk_class(c.X, c.Y, a, cuda_stream, &nl))) return st;
+    }
+    symmetrize_kernel<<<592, 256, 0, s>>>(J, K, n);
+    return cuda_check(cudaGetLastError(), "symmetrize launch");
+  } catch (const std::exception& e) {
+    return fail(MAKO_ERR_OOM, e.what());
+  }
+}
+
+extern "C" mako_status mako_eri_batch(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,
+                                      void* cuda_stream) {
+  try {
+    if (!basis || (nq > 0 && (!quartets || !out))) return fail(MAKO_ERR_INVALID, "NULL argument");
+    if (nq < 0) return fail(MAKO_ERR_INVALID, "nq < 0");
+    int dev = -1;
+    cudaGetDevice(&dev);
+    if (dev != basis->device) return fail(MAKO_ERR_STATE, "basis belongs to another CUDA device");
+    size_t total = 0;
+    for (int q = 0; q < nq; ++q) {
+      size_t sz = 1;
+      for (int k = 0; k < 4; ++k) {
+        int sh = quartets[4 * q + k];
+        if (sh < 0 || sh >= basis->nshell) return fail(MAKO_ERR_INVALID, "shell index out of range");
+        sz *= nsph(basis->l[sh]);
+      }
+      total += sz;
+    }
+    if (total != out_len) return fail(MAKO_ERR_INVALID, "out_len does not match the total block size");
+    if (nq == 0) return MAKO_OK;
+    // canonicalise; one temporary pair per (bra or ket) occurrence
+    std::vector<int> A[NBUCKET], Bs[NBUCKET];
+    struct Item { int X, Y, P, R, flag; long long off; };
+    std::vector<Item> items(nq);
+    size_t off = 0;
+    for (int q = 0; q < nq; ++q) {
+      int u[4] = {quartets[4 * q], quartets[4 * q + 1], quartets[4 * q + 2], quartets[4 * q + 3]};
+      int flag = 0;
+      int ba = u[0], bb = u[1], ka = u[2], kb = u[3];
+      if (basis->l[ba] < basis->l[bb]) { std::swap(ba, bb); flag |= 1; }
+      if (basis->l[ka] < basis->l[kb]) { std::swap(ka, kb); flag |= 2; }
+      int X = bucket_of(basis->l[ba], basis->l[bb]), Y = bucket_of(basis->l[ka], basis->l[kb]);
+      if (X < Y) { std::swap(ba, ka); std::swap(bb, kb); std::swap(X, Y); flag |= 4; }
+      Item& it = items[q];
+      it.X = X; it.Y = Y; it.flag = flag; it.off = (long long)off;
+      it.P = (int)A[X].size(); A[X].push_back(ba); Bs[X].push_back(bb);
+      it.R = (int)A[Y].size(); A[Y].push_back(ka); Bs[Y].push_back(kb);
+      size_t sz = 1;
+      for (int k = 0; k < 4; ++k) sz *= nsph(basis->l[u[k]]);
+      off += sz;
+    }
+    PairSet set;
+    mako_status st;
+    if ((st = build_pair_set(basis, A, Bs, set, cuda_stream))) return st;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    std::vector<std::unique_ptr<DevBuf>> keep;
+    for (int X = 0; X < NBUCKET; ++X)
+      for (int Y = 0; Y <= X; ++Y) {
+        std::vector<int> qb, qk, qf;
+        std::vector<long long> qo;
+        for (auto& it : items)
+          if (it.X == X && it.Y == Y) { qb.push_back(it.P); qk.push_back(it.R); qf.push_back(it.flag); qo.push_back(it.off); }
+        if (qb.empty()) continue;
+        for (int k = 0; k < 4; ++k) keep.emplace_back(new DevBuf);
+        DevBuf& d1 = *keep[keep.size() - 4];
+        DevBuf& d2 = *keep[keep.size() - 3];
+        DevBuf& d3 = *keep[keep.size() - 2];
+        DevBuf& d4 = *keep[keep.size() - 1];
+        if ((st = upload(d1, qb)) || (st = upload(d2, qk)) || (st = upload(d3, qf)) || (st = upload(d4, qo))) return st;
+        BatchArgs a{};
+        a.bra = set.b[X].view();
+        a.ket = set.b[Y].view();
+        a.nq = (int)qb.size();
+        a.qbra = d1.as<int>(); a.qket = d2.as<int>(); a.qflag = d3.as<int>(); a.qout = d4.as<long long>();
+        a.out = out;
+        a.boys = basis->d_boys.as<double>();
+        a.diag = 0;
+        if ((st = launch_batch_class(X, Y, a, cuda_stream))) return st;
+      }
+    return cuda_check(cudaStreamSynchronize(s), "eri_batch sync");
+  } catch (const std::exception& e) {
+    return fail(MAKO_ERR_OOM, e.what());
+  }
+}
+
+extern "C" mako_status mako_boys(int n, const double* T, int mmax, double* out, void* cuda_stream) {
+  if (n < 0 || (n > 0 && (!T || !out)) || mmax < 0 || mmax > 4 * LMAX) return fail(MAKO_ERR_INVALID, "bad args");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(MAKO_ERR_CUDA, "no CUDA device");
+  if (n == 0) return MAKO_OK;
+  static DevBuf tab;
+  static int tab_dev = -1;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (tab_dev != dev) {
+    std::vector<double> h;
+    boys_table(h);
+    mako_status st = upload(tab, h);
+    if (st) return st;
+    tab_dev = dev;
+  }
+  boys_kernel<<<(n + 127) / 128, 128, 0, (cudaStream_t)cuda_stream>>>(n, T, out, tab.as<double>(), mmax);
+  return cuda_check(cudaGetLastError(), "boys launch");
+}

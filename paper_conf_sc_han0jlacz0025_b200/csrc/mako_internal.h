@@ -1,0 +1,96 @@
+// mako_internal.h -- shared internal definitions of libmako (product path only).
+//
+// Hermite / Cartesian index conventions, class geometry, device-side data views.
+// Nothing here is shared with oracle/ (the oracle is an independent implementation).
+#pragma once
+
+#include <cstdint>
+#include <cstddef>
+#include <string>
+#include <vector>
+
+#include "../../include/mako.h"
+
+#ifdef __CUDACC__
+#define MK_HD __host__ __device__
+#else
+#define MK_HD
+#endif
+
+namespace mako {
+
+constexpr int LMAX = MAKO_LMAX;
+constexpr int NBUCKET = (LMAX + 1) * (LMAX + 2) / 2;  // (la >= lb) pair classes: ss ps pp ds dp dd fs fp fd ff
+
+// number of Hermite (or Cartesian) tuples (t,u,v) with t+u+v <= L
+MK_HD constexpr int nH(int L) { return L < 0 ? 0 : (L + 1) * (L + 2) * (L + 3) / 6; }
+MK_HD constexpr int ncart(int l) { return (l + 1) * (l + 2) / 2; }
+MK_HD constexpr int nsph(int l) { return 2 * l + 1; }
+// Hermite index: degree-major, then t descending, then u descending.
+MK_HD constexpr int hidx(int t, int u, int v) {
+  return nH(t + u + v - 1) + (u + v) * (u + v + 1) / 2 + v;
+}
+// Cartesian index within a shell of degree l (lx descending, then ly descending): xx xy xz yy yz zz
+MK_HD constexpr int cart_index(int x, int y, int z) { return (y + z) * (y + z + 1) / 2 + z; }
+// pair bucket of (la >= lb)
+MK_HD constexpr int bucket_of(int la, int lb) { return la * (la + 1) / 2 + lb; }
+
+// Boys table: Taylor grid, F_m(T_k) for T_k = k * BOYS_H, k = 0..BOYS_NGRID-1, m = 0..BOYS_MMAX
+constexpr double BOYS_H = 1.0 / 32.0;
+constexpr double BOYS_TMAX = 40.0;
+constexpr int BOYS_NGRID = 1281;      // T_k up to 40
+constexpr int BOYS_MMAX = 24;         // supports L + 6 <= 24
+constexpr int BOYS_NM = BOYS_MMAX + 1;
+constexpr int BOYS_TAYLOR = 7;        // Taylor terms (|dT| <= 1/64 -> truncation < 5e-17 relative)
+
+// primitive-pair screening (reading R7)
+constexpr double PRIM_PAIR_EPS = 1e-18;
+
+// ---------------------------------------------------------------------------
+// Device view of one bucket of a pair set (all device pointers)
+// ---------------------------------------------------------------------------
+struct PairView {
+  int n;                 // pairs in the bucket
+  int la, lb;
+  const int* shA;        // [n] shell with the higher l (la >= lb)
+  const int* shB;        // [n]
+  const double* Q;       // [n] Schwarz factors (may be null during Schwarz computation)
+  const int* poff;       // [n+1] primitive-pair offsets
+  const double* pdat;    // [nprim][4]: p, Px, Py, Pz
+  const double* Ebra;    // [nprim][nab][nHab]  E~ with spherical transform, coefficients, 1/p folded
+  const double* Eket;    // [nprim][nHab][nab]  (-1)^{|q|} E~^T
+};
+
+// arguments of a J/K class launch
+struct JKArgs {
+  PairView bra, ket;
+  int same_bucket;
+  long long task_begin, task_end;   // shard range of this class's task index space
+  const long long* task_off;        // [nbra+1] task prefix per bra pair
+  const int* nket;                  // [nbra] kets per bra (prefix of the Q-sorted ket bucket)
+  int nbra;
+  int KT;                           // kets per task
+  unsigned long long* counter;      // dynamic task counter (zeroed before launch)
+  const double* D;
+  double* J;                        // accumulators (symmetrised afterwards)
+  double* K;
+  int nbf;
+  const int* ao;                    // [nshell] AO offsets
+  double thresh;
+  const double* boys;               // Boys table
+};
+
+// arguments of a store/diag class launch (eri_batch, Schwarz)
+struct BatchArgs {
+  PairView bra, ket;
+  int nq;
+  const int* qbra;        // [nq] bra pair index in bucket
+  const int* qket;        // [nq] ket pair index
+  const long long* qout;  // [nq] output offset (store mode) or Q index (diag mode)
+  const int* qflag;       // [nq] bit0 swap a/b, bit1 swap c/d, bit2 swap bra/ket (store mode)
+  double* out;
+  const double* boys;
+  int diag;               // 1 = Schwarz mode: out[qout[i]] = sqrt(max |(ab|ab)|)
+};
+
+}  // namespace mako

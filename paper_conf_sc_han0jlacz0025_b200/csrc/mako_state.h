@@ -1,0 +1,109 @@
+// mako_state.h -- host-side state behind the opaque handles of include/mako.h.
+#pragma once
+
+#include <map>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "mako_internal.h"
+
+namespace mako {
+
+// thread-local error message
+void set_error(const std::string& msg);
+mako_status fail(mako_status st, const std::string& msg);
+const char* last_error_cstr();
+
+// owning device buffer (cudaMalloc / cudaFree)
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  DevBuf() = default;
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  DevBuf(DevBuf&& o) noexcept : p(o.p), bytes(o.bytes) { o.p = nullptr; o.bytes = 0; }
+  DevBuf& operator=(DevBuf&& o) noexcept {
+    if (this != &o) {
+      release();
+      p = o.p; bytes = o.bytes;
+      o.p = nullptr; o.bytes = 0;
+    }
+    return *this;
+  }
+  ~DevBuf();
+  mako_status alloc(size_t nbytes);
+  template <class T> T* as() const { return static_cast<T*>(p); }
+  void release();
+};
+
+// one bucket (la >= lb) of shell pairs with device-resident primitive-pair data
+struct PairBucket {
+  int la = 0, lb = 0;
+  std::vector<int> shA, shB;       // host copies
+  std::vector<double> Q;           // host copy (sorted descending in a screened set)
+  std::vector<int> poff;           // [n+1]
+  DevBuf d_shA, d_shB, d_Q, d_poff, d_pdat, d_Ebra, d_Eket;
+  int n() const { return (int)shA.size(); }
+  PairView view() const;
+};
+
+struct PairSet {
+  PairBucket b[NBUCKET];
+};
+
+// per-class plan for one threshold
+struct ClassPlan {
+  int X = 0, Y = 0;                // bra / ket buckets (X >= Y)
+  long long ntask = 0;             // tasks of the whole class (all shards)
+  long long nquartet = 0;
+  std::vector<int> nket;           // [nbra]
+  std::vector<long long> task_off; // [nbra+1]
+  DevBuf d_nket, d_task_off;
+};
+
+struct Plan {
+  double thresh = -1.0;
+  int KT = 16;
+  std::vector<ClassPlan> cls;      // 55 classes
+};
+
+}  // namespace mako
+
+struct mako_basis_s {
+  int device = 0;
+  int natm = 0;
+  std::vector<int> Z;
+  std::vector<double> axyz;
+  int nshell = 0, nbf = 0, pure = 1;
+  std::vector<int> atom, l, nprim, poff, ao;
+  std::vector<double> sxyz;     // [nshell*3] shell centres
+  std::vector<double> exps, cn; // exponents; coefficient x primitive norm x contraction renorm
+  mako::DevBuf d_ao, d_sxyz, d_l, d_poff, d_exps, d_cn, d_sph, d_boys;
+  std::vector<int> sph_off;     // offset of each l's [2l+1][ncart] table in d_sph
+};
+
+struct mako_pairs_s {
+  mako_basis basis = nullptr;   // not owned; must outlive the pairs
+  double tau = 0.0;
+  mako::PairSet set;
+  mako::Plan plan;
+  mako::DevBuf d_counters;      // [55] task counters
+};
+
+namespace mako {
+// host helpers implemented in basis.cpp
+void spherical_tables(std::vector<double>& tab, std::vector<int>& off);   // recurrence-derived
+void boys_table(std::vector<double>& tab);                                // composite Gauss-Legendre
+// pair-set construction (pairs.cu)
+mako_status build_pair_set(const mako_basis_s* B, const std::vector<int> (&A)[NBUCKET],
+                           const std::vector<int> (&Bsh)[NBUCKET], PairSet& out, void* stream);
+mako_status compute_schwarz(const mako_basis_s* B, PairSet& set, void* stream);
+// class launches (eri_kernels*.cu)
+mako_status launch_jk_class(int X, int Y, const JKArgs& a, void* stream, int* nlaunch);
+mako_status launch_batch_class(int X, int Y, const BatchArgs& a, void* stream);
+// class index (X >= Y) in 0..54
+inline int class_index(int X, int Y) { return X * (X + 1) / 2 + Y; }
+inline int bucket_la(int b) { int la = 0; while ((la + 1) * (la + 2) / 2 <= b) ++la; return la; }
+inline int bucket_lb(int b) { int la = bucket_la(b); return b - la * (la + 1) / 2; }
+}  // namespace mako

@@ -1,0 +1,147 @@
+"""Python API over the C ABI (include/mako.h): Basis, Pairs, build_jk, eri_batch, boys.
+
+PyTorch provides device memory and streams only; every step of the J/K path runs in libmako's
+CUDA kernels.  Device tensors must be float64, contiguous, on the handle's CUDA device.
+"""
+import ctypes
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import check
+
+
+def _i32(a):
+    a = np.ascontiguousarray(a, dtype=np.int32)
+    return a, a.ctypes.data_as(ctypes.POINTER(ctypes.c_int))
+
+
+def _f64(a):
+    a = np.ascontiguousarray(a, dtype=np.float64)
+    return a, a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _dev_ptr(t, name):
+    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+        raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+class Basis:
+    """Gaussian basis on a molecule.  ``shells`` is a mako_inputs.Shells-like
+    object (atom, l, nprim, exps, coefs); ``Z``/``xyz`` the atoms (bohr)."""
+
+    def __init__(self, Z, xyz, shells, pure=True):
+        self._lib = _lib.load()
+        Zc, Zp = _i32(Z)
+        Xc, Xp = _f64(np.asarray(xyz).reshape(-1))
+        a, ap = _i32(shells.atom)
+        l, lp = _i32(shells.l)
+        n, npp = _i32(shells.nprim)
+        e, ep = _f64(shells.exps)
+        c, cp = _f64(shells.coefs)
+        h = ctypes.c_void_p()
+        check(self._lib.mako_basis_create(len(Zc), Zp, Xp, len(l), ap, lp, npp, ep, cp, 1 if pure else 0,
+                                          ctypes.byref(h)))
+        self.handle = h
+        nbf = ctypes.c_int()
+        check(self._lib.mako_basis_nbf(h, ctypes.byref(nbf)))
+        self.nbf = nbf.value
+        self.nshell = len(l)
+        ao = np.zeros(self.nshell + 1, np.int32)
+        check(self._lib.mako_basis_ao_offsets(h, ao.ctypes.data_as(ctypes.POINTER(ctypes.c_int))))
+        self.ao_offsets = ao
+        self.l = l.copy()
+
+    @classmethod
+    def from_molecule(cls, mol, shells):
+        return cls(mol.Z, mol.xyz_bohr, shells)
+
+    def close(self):
+        if getattr(self, "handle", None):
+            self._lib.mako_basis_destroy(self.handle)
+            self.handle = None
+
+    __del__ = close
+
+
+class Pairs:
+    """Screened shell-pair data (Schwarz threshold tau), device resident."""
+
+    def __init__(self, basis, tau=1e-12, stream=None):
+        self._lib = basis._lib
+        self.basis = basis  # keeps the basis alive
+        self.tau = tau
+        h = ctypes.c_void_p()
+        check(self._lib.mako_shellpairs_screen(basis.handle, float(tau), _stream_ptr(stream), ctypes.byref(h)))
+        self.handle = h
+
+    def stats(self, thresh=None):
+        a, b, c = ctypes.c_longlong(), ctypes.c_longlong(), ctypes.c_longlong()
+        check(self._lib.mako_pairs_stats(self.handle, float(self.tau if thresh is None else thresh), ctypes.byref(a),
+                                         ctypes.byref(b), ctypes.byref(c)))
+        return {"pairs": a.value, "prim_pairs": b.value, "quartets": c.value}
+
+    def flops(self, thresh=None, shard=0, nshards=1):
+        f, q, pq = ctypes.c_double(), ctypes.c_longlong(), ctypes.c_longlong()
+        check(self._lib.mako_pairs_flops(self.handle, float(self.tau if thresh is None else thresh), shard, nshards,
+                                         ctypes.byref(f), ctypes.byref(q), ctypes.byref(pq)))
+        return {"gemm_flops": f.value, "quartets": q.value, "prim_quartets": pq.value}
+
+    def launches(self, thresh=None, shard=0, nshards=1):
+        n = ctypes.c_int()
+        check(self._lib.mako_build_jk_launches(self.handle, float(self.tau if thresh is None else thresh), shard,
+                                               nshards, ctypes.byref(n)))
+        return n.value
+
+    def close(self):
+        if getattr(self, "handle", None):
+            self._lib.mako_pairs_destroy(self.handle)
+            self.handle = None
+
+    __del__ = close
+
+
+def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=None):
+    """J_{mn} = sum (mn|ls) D_ls, K_{ml} = sum (mn|ls) D_ns on the GPU (north_star).  Async on `stream`."""
+    n = pairs.basis.nbf
+    if D.shape != (n, n):
+        raise ValueError(f"D must be {n}x{n}")
+    if J is None:
+        J = torch.empty_like(D)
+    if K is None:
+        K = torch.empty_like(D)
+    check(pairs._lib.mako_build_jk(pairs.handle, _dev_ptr(D, "D"), float(pairs.tau if thresh is None else thresh),
+                                   _dev_ptr(J, "J"), _dev_ptr(K, "K"), int(shard), int(nshards), _stream_ptr(stream)))
+    return J, K
+
+
+def eri_batch(basis, quartets, stream=None, device=None):
+    """Shell-quartet ERI blocks (test entry).  Returns a list of numpy-shaped torch tensors on the GPU."""
+    q, qp = _i32(np.asarray(quartets).reshape(-1, 4))
+    # out-of-range shells are left to the C ABI to reject (MAKO_ERR_INVALID)
+    nf = lambda s: 2 * int(basis.l[s]) + 1 if 0 <= s < basis.nshell else 0
+    sizes = [int(np.prod([nf(s) for s in row])) for row in q]
+    out = torch.empty(sum(sizes), dtype=torch.float64, device=device or "cuda")
+    check(basis._lib.mako_eri_batch(basis.handle, len(q), qp, _dev_ptr(out, "out"), out.numel(), _stream_ptr(stream)))
+    res, o = [], 0
+    for row, s in zip(q, sizes):
+        res.append(out[o:o + s].view(*[2 * basis.l[x] + 1 for x in row]))
+        o += s
+    return res
+
+
+def boys(T, mmax, stream=None):
+    """Device Boys evaluator of the hot path: T (CUDA float64 [n]) -> [n, mmax+1]."""
+    lib = _lib.load()
+    T = T.contiguous()
+    out = torch.empty((T.numel(), mmax + 1), dtype=torch.float64, device=T.device)
+    check(lib.mako_boys(T.numel(), _dev_ptr(T, "T"), int(mmax), _dev_ptr(out, "out"), _stream_ptr(stream)))
+    return out
