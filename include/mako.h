@@ -118,6 +118,23 @@ mako_status mako_build_jk(mako_pairs pairs, const double* D, double thresh, doub
 /* Number of CUDA kernels one mako_build_jk call launches for these arguments (for bench accounting). */
 mako_status mako_build_jk_launches(mako_pairs pairs, double thresh, int shard, int nshards, int* n_launches);
 
+/* Number of angular-momentum classes (bra bucket X >= ket bucket Y over the 10 (la>=lb) pair
+ * buckets ss ps pp ds dp dd fs fp fd ff): class index c = X(X+1)/2 + Y. */
+#define MAKO_NCLASS 55
+
+/* Per-class algorithmic GEMM FLOPs (same definition as mako_pairs_flops) and quartet counts of
+ * shard `shard`/`nshards` at thresh.  flops[MAKO_NCLASS], quartets[MAKO_NCLASS] (HOST, either NULL). */
+mako_status mako_pairs_class_flops(mako_pairs pairs, double thresh, int shard, int nshards, double* flops,
+                                   long long* quartets);
+
+/* Measurement hooks.  mako_profile_enable(pairs, 1) resets and starts recording a CUDA event pair
+ * around every class-kernel launch of subsequent mako_build_jk calls (on their stream);
+ * mako_profile_read synchronises those events and returns, per class index, the summed kernel
+ * milliseconds and the number of launches since enable (HOST arrays of MAKO_NCLASS, either NULL).
+ * enable = 0 stops recording and frees the events. */
+mako_status mako_profile_enable(mako_pairs pairs, int enable);
+mako_status mako_profile_read(mako_pairs pairs, double* ms, long long* launches);
+
 /* Test entry: nq shell quartets, quartets[4*q .. 4*q+3] = shell indices (a,b,c,d) in
  * any order (HOST array).  out (DEVICE, FP64) receives the blocks (ab|cd) concatenated in quartet
  * order, each laid out [n_a][n_b][n_c][n_d] in the AO order of each shell.  out_len (elements) must

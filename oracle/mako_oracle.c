@@ -533,15 +533,20 @@ static void digest(const basis_t* B, int a, int b, int c, int d, const double* b
 /* Screened J/K over canonical shell quartets (a>=b, c>=d, ab>=cd); keep iff Q_ab Q_cd >= tau.
    shard/nshards: only canonical bra pairs with (pair_index % nshards == shard) are evaluated
    (an oracle-side sample; the GPU library's own shard partition is not replicated here).
+   Qin: optional precomputed Schwarz table (orc_schwarz), NULL to compute it here.
    J, K: [nbf][nbf] outputs (overwritten), final symmetrised values. */
-int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, double* Jout, double* Kout) {
+int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, const double* Qin, double* Jout,
+           double* Kout) {
   BASIS_INIT(B);
   if (nshards < 1 || shard < 0 || shard >= nshards || tau < 0) { basis_free(&B); return 1; }
   int N = B.nbf;
   double* Q = (double*)malloc(sizeof(double) * nshell * nshell);
-  basis_free(&B);
-  orc_schwarz(nshell, l, nprim, xyz, exps, coefs, pure, Q);
-  if (basis_init(&B, nshell, l, nprim, xyz, exps, coefs, pure)) return 2;
+  if (Qin) memcpy(Q, Qin, sizeof(double) * nshell * nshell);
+  else {
+    basis_free(&B);
+    orc_schwarz(nshell, l, nprim, xyz, exps, coefs, pure, Q);
+    if (basis_init(&B, nshell, l, nprim, xyz, exps, coefs, pure)) return 2;
+  }
   int npair = nshell * (nshell + 1) / 2;
   int* pa = (int*)malloc(sizeof(int) * npair);
   int* pb = (int*)malloc(sizeof(int) * npair);

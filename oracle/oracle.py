@@ -95,13 +95,17 @@ def schwarz(sh, pure=True):
     return Q
 
 
-def jk(sh, D, tau=0.0, shard=0, nshards=1, pure=True):
+def jk(sh, D, tau=0.0, shard=0, nshards=1, pure=True, Q=None):
     keep, args = _basis_args(sh, pure)
     N = sh.nbf(pure)
     D = np.ascontiguousarray(D, dtype=np.float64)
     assert D.shape == (N, N)
     J = np.zeros((N, N)); K = np.zeros((N, N))
-    _check(_get().orc_jk(*args, _d(D), ctypes.c_double(tau), shard, nshards, _d(J), _d(K)), "jk")
+    Qp = None
+    if Q is not None:
+        Q = np.ascontiguousarray(Q, dtype=np.float64)
+        Qp = _d(Q)
+    _check(_get().orc_jk(*args, _d(D), ctypes.c_double(tau), shard, nshards, Qp, _d(J), _d(K)), "jk")
     return J, K
 
 

@@ -10,13 +10,15 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libmako.so")
 
 MAKO_OK = 0
+NCLASS = 55
 STATUS = {0: "MAKO_OK", 1: "MAKO_ERR_INVALID", 2: "MAKO_ERR_UNSUPPORTED", 3: "MAKO_ERR_CUDA", 4: "MAKO_ERR_OOM",
           5: "MAKO_ERR_STATE"}
 
 # every symbol include/mako.h declares (checked by tests/test_abi.py)
 EXPORTS = ["mako_basis_create", "mako_basis_nbf", "mako_basis_nshell", "mako_basis_ao_offsets", "mako_basis_destroy",
            "mako_shellpairs_screen", "mako_pairs_stats", "mako_pairs_flops", "mako_pairs_destroy", "mako_build_jk",
-           "mako_build_jk_launches", "mako_eri_batch", "mako_boys", "mako_last_error", "mako_version"]
+           "mako_build_jk_launches", "mako_eri_batch", "mako_boys", "mako_last_error", "mako_version",
+           "mako_pairs_class_flops", "mako_profile_enable", "mako_profile_read"]
 
 
 class MakoError(RuntimeError):
@@ -57,6 +59,10 @@ def load():
         "mako_build_jk_launches": ([_vp, ctypes.c_double, ctypes.c_int, ctypes.c_int, _ip], ctypes.c_int),
         "mako_eri_batch": ([_vp, ctypes.c_int, _ip, _vp, ctypes.c_size_t, _vp], ctypes.c_int),
         "mako_boys": ([ctypes.c_int, _vp, ctypes.c_int, _vp, _vp], ctypes.c_int),
+        "mako_pairs_class_flops": ([_vp, ctypes.c_double, ctypes.c_int, ctypes.c_int, _dp, ctypes.POINTER(_ll)],
+                                   ctypes.c_int),
+        "mako_profile_enable": ([_vp, ctypes.c_int], ctypes.c_int),
+        "mako_profile_read": ([_vp, _dp, ctypes.POINTER(_ll)], ctypes.c_int),
         "mako_last_error": ([], ctypes.c_char_p),
         "mako_version": ([], ctypes.c_char_p),
     }

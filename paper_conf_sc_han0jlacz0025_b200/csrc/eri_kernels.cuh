@@ -21,6 +21,7 @@ int jk_blocks_per_sm();
 
 #ifdef MAKO_DEFINE_KERNELS
 #include "eri_core.cuh"
+#include "eri_tpq.cuh"
 
 namespace mako {
 
@@ -142,9 +143,13 @@ int jk_blocks_per_sm() {
   constexpr size_t smem = cta_smem_bytes<C>();
   static int cached = -1;
   if (cached < 0) {
-    if (set_smem_attr<X, Y>((const void*)jk_kernel<X, Y>, smem)) return 1;
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel<X, Y>, CTA_THREADS, smem);
+    if constexpr (use_tpq(X, Y)) {
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, tpq_jk_kernel<X, Y>, CTA_THREADS, 0);
+    } else {
+      if (set_smem_attr<X, Y>((const void*)jk_kernel<X, Y>, smem)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel<X, Y>, CTA_THREADS, smem);
+    }
     cached = nb < 1 ? 1 : nb;
   }
   return cached;
@@ -163,7 +168,10 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   long long want = (ntask + CTA_WARPS - 1) / CTA_WARPS;
   long long cap = (long long)nsm * bps;
   const int grid = (int)(want < cap ? want : cap);
-  jk_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
+  if constexpr (use_tpq(X, Y))
+    tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, (cudaStream_t)stream>>>(a);
+  else
+    jk_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("jk_kernel launch: ") + cudaGetErrorString(e));
   if (nlaunch) ++*nlaunch;

@@ -1,0 +1,251 @@
+// eri_tpq.cuh -- lane-per-ket register kernel for the low angular-momentum classes.
+//
+// The paper's "striped layout" (S3.1.2: one thread per shell quartet, each
+// parameter strided by the batch) taken to its end for classes whose whole MMD state fits in
+// registers: a warp owns one bra pair and 32 consecutive kets of its Q-sorted prefix; lane i
+// evaluates quartet (bra | ket_i) completely in registers:
+//   Boys F_m (a4) -> R^{(0)}_{tuv} by Eq. 5 fully unrolled at compile time (a5) ->
+//   W[p][cd] = sum_q R_{p+q} (-1)^{|q|} E~_cd[q][cd]  then  V[ab][cd] += E~_ab[ab][p] W[p][cd]
+//   (Eq. 7 with the cheaper contraction order for a low-l ket; the bra E~ is warp-uniform) ->
+//   digestion (a9): J_ab by warp reduction, J_cd / K blocks by FP64 atomics from each lane.
+#pragma once
+
+#include <utility>
+
+#include "eri_core.cuh"
+
+namespace mako {
+
+// compile-time Hermite decode (degree-major, t desc, u desc)
+MK_HD constexpr int hd_k(int e) { int k = 0; while (nH(k) <= e) ++k; return k; }
+MK_HD constexpr int hd_s(int e) {
+  int r = e - nH(hd_k(e) - 1), s = 0;
+  while ((s + 1) * (s + 2) / 2 <= r) ++s;
+  return s;
+}
+MK_HD constexpr int hd_v(int e) { return e - nH(hd_k(e) - 1) - hd_s(e) * (hd_s(e) + 1) / 2; }
+MK_HD constexpr int hd_u(int e) { return hd_s(e) - hd_v(e); }
+MK_HD constexpr int hd_t(int e) { return hd_k(e) - hd_s(e); }
+MK_HD constexpr int r_dir(int e) { return hd_t(e) > 0 ? 0 : (hd_u(e) > 0 ? 1 : 2); }
+MK_HD constexpr int r_n(int e) { return r_dir(e) == 0 ? hd_t(e) : (r_dir(e) == 1 ? hd_u(e) : hd_v(e)); }
+MK_HD constexpr int r_src(int e, int m) {  // index of e - m * 1_dir
+  return r_dir(e) == 0 ? hidx(hd_t(e) - m, hd_u(e), hd_v(e))
+                       : (r_dir(e) == 1 ? hidx(hd_t(e), hd_u(e) - m, hd_v(e)) : hidx(hd_t(e), hd_u(e), hd_v(e) - m));
+}
+MK_HD constexpr int h_sum(int p, int q) {
+  return hidx(hd_t(p) + hd_t(q), hd_u(p) + hd_u(q), hd_v(p) + hd_v(q));
+}
+
+template <int B, int E, class F>
+__device__ __forceinline__ void static_for(F&& f) {
+  if constexpr (B < E) {
+    f(std::integral_constant<int, B>{});
+    static_for<B + 1, E>(f);
+  }
+}
+
+// one level of the in-place R recursion: entries E, E-1, ..., 1 (descending = degree-descending,
+// so every source of level n+1 is still unmodified when read)
+template <int E>
+__device__ __forceinline__ void r_level(double* R, double X, double Y, double Z) {
+  if constexpr (E >= 1) {
+    constexpr int dir = r_dir(E), n = r_n(E), s1 = r_src(E, 1);
+    const double x = dir == 0 ? X : (dir == 1 ? Y : Z);
+    if constexpr (n >= 2) {
+      constexpr int s2 = r_src(E, 2);
+      R[E] = fma((double)(n - 1), R[s2], x * R[s1]);
+    } else {
+      R[E] = x * R[s1];
+    }
+    r_level<E - 1>(R, X, Y, Z);
+  }
+}
+
+template <int L, int N>
+__device__ __forceinline__ void r_levels(double* R, const double* F, double X, double Y, double Z) {
+  if constexpr (N >= 0) {
+    r_level<nH(L - N) - 1>(R, X, Y, Z);
+    R[0] = F[N];
+    r_levels<L, N - 1>(R, F, X, Y, Z);
+  }
+}
+
+// Boys + R^{(0)} into registers (R[nH(L)]), seeds scaled by 2 pi^{5/2}/sqrt(p+q) (-2 rho)^n
+template <int L>
+__device__ __forceinline__ void r_regs(double p, double Px, double Py, double Pz, double q, double Qx, double Qy,
+                                       double Qz, const double* __restrict__ btab, double (&R)[nH(L)]) {
+  const double pq = p + q, rho = p * q / pq;
+  const double X = Px - Qx, Y = Py - Qy, Z = Pz - Qz;
+  double F[L + 1];
+  boys_eval<L>(rho * (X * X + Y * Y + Z * Z), btab, F);
+  double s = TWO_PI_52 * rsqrt(pq);
+  const double m2r = -2.0 * rho;
+#pragma unroll
+  for (int n = 0; n <= L; ++n) {
+    F[n] *= s;
+    s *= m2r;
+  }
+  R[0] = F[L];
+  r_levels<L, L - 1>(R, F, X, Y, Z);
+}
+
+// Persistent lane-per-ket kernel (JKArgs.KT must be 32).
+template <int X, int Y>
+__global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
+  using C = ClsXY<X, Y>;
+  constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
+  constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND;
+  const int lane = threadIdx.x & 31;
+  for (;;) {
+    unsigned long long tk = 0;
+    if (lane == 0) tk = atomicAdd(a.counter, 1ull);
+    tk = __shfl_sync(0xffffffffu, tk, 0);
+    const long long task = a.task_begin + (long long)tk;
+    if (task >= a.task_end) break;
+    int lo = 0, hi = a.nbra - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (__ldg(a.task_off + mid) <= task) lo = mid; else hi = mid - 1;
+    }
+    const int P = lo;
+    const int r0 = (int)(task - __ldg(a.task_off + P)) * 32;
+    const int r1 = min(r0 + 32, __ldg(a.nket + P));
+    const int R = r0 + lane;
+    const double QP = __ldg(a.bra.Q + P);
+    const bool active = R < r1 && QP * __ldg(a.ket.Q + min(R, r1 - 1)) >= a.thresh;
+    const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
+    const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
+    const int b0 = __ldg(a.bra.poff + P), b1 = __ldg(a.bra.poff + P + 1);
+    double V[NAB][NCD];
+#pragma unroll
+    for (int i = 0; i < NAB; ++i)
+#pragma unroll
+      for (int j = 0; j < NCD; ++j) V[i][j] = 0.0;
+    int sc = 0, sd = 0;
+    if (active) {
+      sc = __ldg(a.ket.shA + R);
+      sd = __ldg(a.ket.shB + R);
+      const int k0 = __ldg(a.ket.poff + R), k1 = __ldg(a.ket.poff + R + 1);
+      for (int kl = k0; kl < k1; ++kl) {
+        const double q = __ldg(a.ket.pdat + 4 * kl), Qx = __ldg(a.ket.pdat + 4 * kl + 1),
+                     Qy = __ldg(a.ket.pdat + 4 * kl + 2), Qz = __ldg(a.ket.pdat + 4 * kl + 3);
+        // signed ket E~^T [q][cd]
+        double Ek[NHCD][NCD];
+        const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
+#pragma unroll
+        for (int h = 0; h < NHCD; ++h)
+#pragma unroll
+          for (int j = 0; j < NCD; ++j) Ek[h][j] = __ldg(ek + h * NCD + j);
+        for (int ij = b0; ij < b1; ++ij) {
+          const double p = __ldg(a.bra.pdat + 4 * ij), Px = __ldg(a.bra.pdat + 4 * ij + 1),
+                       Py = __ldg(a.bra.pdat + 4 * ij + 2), Pz = __ldg(a.bra.pdat + 4 * ij + 3);
+          double Rr[nH(L)];
+          r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
+          const double* __restrict__ eb = a.bra.Ebra + (size_t)ij * (NAB * NHAB);
+          static_for<0, NHAB>([&](auto pc) {
+            constexpr int pp = decltype(pc)::value;
+            double W[NCD];
+#pragma unroll
+            for (int j = 0; j < NCD; ++j) W[j] = 0.0;
+            static_for<0, NHCD>([&](auto qc) {
+              constexpr int qq = decltype(qc)::value;
+              constexpr int hs = h_sum(pp, qq);
+#pragma unroll
+              for (int j = 0; j < NCD; ++j) W[j] = fma(Rr[hs], Ek[qq][j], W[j]);
+            });
+#pragma unroll
+            for (int i = 0; i < NAB; ++i) {
+              const double e = __ldg(eb + i * NHAB + pp);
+#pragma unroll
+              for (int j = 0; j < NCD; ++j) V[i][j] = fma(e, W[j], V[i][j]);
+            }
+          });
+        }
+      }
+    }
+    // ---- digestion (a9) ----
+    double deg = 1.0;
+    if (sa == sb) deg *= 0.5;
+    if (sc == sd) deg *= 0.5;
+    if (a.same_bucket && P == R) deg *= 0.5;
+    if (!active) deg = 0.0;
+    const double* __restrict__ Dm = a.D;
+    const size_t n = (size_t)a.nbf;
+    const int oc = active ? __ldg(a.ao + sc) : 0, od = active ? __ldg(a.ao + sd) : 0;
+    // J_ab: per-lane deg-weighted partial, warp reduction over the 32 kets, one atomic per element
+#pragma unroll
+    for (int i = 0; i < NAB; ++i) {
+      double s = 0.0;
+      if (active) {
+#pragma unroll
+        for (int k = 0; k < NC; ++k)
+#pragma unroll
+          for (int l = 0; l < ND; ++l) s = fma(V[i][k * ND + l], __ldg(Dm + (oc + k) * n + od + l), s);
+      }
+      s *= deg;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+      if (lane == 0) atomicAdd(a.J + (oa + i / NB) * n + ob + i % NB, 2.0 * s);
+    }
+    if (!active) continue;
+    // J_cd
+#pragma unroll
+    for (int k = 0; k < NC; ++k)
+#pragma unroll
+      for (int l = 0; l < ND; ++l) {
+        double s = 0.0;
+#pragma unroll
+        for (int i = 0; i < NA; ++i)
+#pragma unroll
+          for (int j = 0; j < NB; ++j) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (oa + i) * n + ob + j), s);
+        atomicAdd(a.J + (oc + k) * n + od + l, 2.0 * deg * s);
+      }
+    // K_ac += v D_bd ; K_ad += v D_bc ; K_bc += v D_ad ; K_bd += v D_ac
+#pragma unroll
+    for (int i = 0; i < NA; ++i)
+#pragma unroll
+      for (int k = 0; k < NC; ++k) {
+        double s = 0.0;
+#pragma unroll
+        for (int j = 0; j < NB; ++j)
+#pragma unroll
+          for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (ob + j) * n + od + l), s);
+        atomicAdd(a.K + (oa + i) * n + oc + k, deg * s);
+      }
+#pragma unroll
+    for (int i = 0; i < NA; ++i)
+#pragma unroll
+      for (int l = 0; l < ND; ++l) {
+        double s = 0.0;
+#pragma unroll
+        for (int j = 0; j < NB; ++j)
+#pragma unroll
+          for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (ob + j) * n + oc + k), s);
+        atomicAdd(a.K + (oa + i) * n + od + l, deg * s);
+      }
+#pragma unroll
+    for (int j = 0; j < NB; ++j)
+#pragma unroll
+      for (int k = 0; k < NC; ++k) {
+        double s = 0.0;
+#pragma unroll
+        for (int i = 0; i < NA; ++i)
+#pragma unroll
+          for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (oa + i) * n + od + l), s);
+        atomicAdd(a.K + (ob + j) * n + oc + k, deg * s);
+      }
+#pragma unroll
+    for (int j = 0; j < NB; ++j)
+#pragma unroll
+      for (int l = 0; l < ND; ++l) {
+        double s = 0.0;
+#pragma unroll
+        for (int i = 0; i < NA; ++i)
+#pragma unroll
+          for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (oa + i) * n + oc + k), s);
+        atomicAdd(a.K + (ob + j) * n + od + l, deg * s);
+      }
+  }
+}
+
+}  // namespace mako

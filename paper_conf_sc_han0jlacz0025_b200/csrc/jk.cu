@@ -71,6 +71,7 @@ static mako_status ensure_plan(mako_pairs P, double thresh) {
       ClassPlan& c = pl.cls[class_index(X, Y)];
       c.X = X;
       c.Y = Y;
+      c.KT = class_kt(X, Y);
       const PairBucket& bx = P->set.b[X];
       const PairBucket& by = P->set.b[Y];
       const int nbra = bx.n();
@@ -81,7 +82,7 @@ static mako_status ensure_plan(mako_pairs P, double thresh) {
         if (X == Y) nk = std::min(nk, p + 1);
         c.nket[p] = nk;
         c.nquartet += nk;
-        c.task_off[p + 1] = c.task_off[p] + (nk + pl.KT - 1) / pl.KT;
+        c.task_off[p + 1] = c.task_off[p] + (nk + c.KT - 1) / c.KT;
       }
       c.ntask = c.task_off[nbra];
       mako_status st;
@@ -159,45 +160,117 @@ extern "C" mako_status mako_pairs_stats(mako_pairs p, double thresh, long long* 
   }
 }
 
+// per-class algorithmic GEMM FLOPs / quartets / primitive quartets of one shard
+static mako_status class_flops(mako_pairs p, double thresh, int shard, int nshards, std::vector<double>& fl,
+                               std::vector<long long>& nq, std::vector<long long>& npq) {
+  mako_status st;
+  if ((st = check_pairs(p))) return st;
+  if (!(thresh >= 0) || nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "bad args");
+  thresh = std::max(thresh, p->tau);
+  if ((st = ensure_plan(p, thresh))) return st;
+  const int NC = NBUCKET * (NBUCKET + 1) / 2;
+  fl.assign(NC, 0.0);
+  nq.assign(NC, 0);
+  npq.assign(NC, 0);
+  for (auto& c : p->plan.cls) {
+    const int KT = c.KT;
+    const int ci = class_index(c.X, c.Y);
+    const PairBucket& bx = p->set.b[c.X];
+    const PairBucket& by = p->set.b[c.Y];
+    const int la = bx.la, lb = bx.lb, lc = by.la, ld = by.lb;
+    const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
+    const double hab = nH(la + lb), hcd = nH(lc + ld);
+    const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
+    // ket prefix of bra P restricted to this shard's tasks; by.poff is the prefix sum of K_CD
+    for (int P = 0; P < (int)c.nket.size(); ++P) {
+      const long long a0 = c.task_off[P], a1 = c.task_off[P + 1];
+      if (a1 <= t0 || a0 >= t1) continue;
+      const long long KAB = bx.poff[P + 1] - bx.poff[P];
+      const int r0 = (int)(std::max(a0, t0) - a0) * KT;
+      const int r1 = std::min((int)(std::min(a1, t1) - a0) * KT, c.nket[P]);
+      if (r1 <= r0) continue;
+      const long long sumK = by.poff[r1] - by.poff[r0];
+      fl[ci] += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)sumK * 2.0 * nab * hcd * ncd;
+      nq[ci] += r1 - r0;
+      npq[ci] += KAB * sumK;
+    }
+  }
+  return MAKO_OK;
+}
+
 extern "C" mako_status mako_pairs_flops(mako_pairs p, double thresh, int shard, int nshards, double* gemm_flops,
                                         long long* n_quartets, long long* n_prim_quartets) {
   try {
-    mako_status st;
-    if ((st = check_pairs(p))) return st;
-    if (!(thresh >= 0) || nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "bad args");
-    thresh = std::max(thresh, p->tau);
-    if ((st = ensure_plan(p, thresh))) return st;
-    double fl = 0;
-    long long nq = 0, npq = 0;
-    const int KT = p->plan.KT;
-    for (auto& c : p->plan.cls) {
-      const PairBucket& bx = p->set.b[c.X];
-      const PairBucket& by = p->set.b[c.Y];
-      const int la = bx.la, lb = bx.lb, lc = by.la, ld = by.lb;
-      const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
-      const double hab = nH(la + lb), hcd = nH(lc + ld);
-      const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
-      // ket prefix of bra P restricted to this shard's tasks; by.poff is the prefix sum of K_CD
-      for (int P = 0; P < (int)c.nket.size(); ++P) {
-        const long long a0 = c.task_off[P], a1 = c.task_off[P + 1];
-        if (a1 <= t0 || a0 >= t1) continue;
-        const long long KAB = bx.poff[P + 1] - bx.poff[P];
-        const int r0 = (int)(std::max(a0, t0) - a0) * KT;
-        const int r1 = std::min((int)(std::min(a1, t1) - a0) * KT, c.nket[P]);
-        if (r1 <= r0) continue;
-        const long long sumK = by.poff[r1] - by.poff[r0];
-        fl += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)sumK * 2.0 * nab * hcd * ncd;
-        nq += r1 - r0;
-        npq += KAB * sumK;
-      }
-    }
-    if (gemm_flops) *gemm_flops = fl;
-    if (n_quartets) *n_quartets = nq;
-    if (n_prim_quartets) *n_prim_quartets = npq;
+    std::vector<double> fl;
+    std::vector<long long> nq, npq;
+    mako_status st = class_flops(p, thresh, shard, nshards, fl, nq, npq);
+    if (st) return st;
+    double f = 0;
+    long long a = 0, b = 0;
+    for (size_t i = 0; i < fl.size(); ++i) { f += fl[i]; a += nq[i]; b += npq[i]; }
+    if (gemm_flops) *gemm_flops = f;
+    if (n_quartets) *n_quartets = a;
+    if (n_prim_quartets) *n_prim_quartets = b;
     return MAKO_OK;
   } catch (const std::exception& e) {
     return fail(MAKO_ERR_OOM, e.what());
   }
+}
+
+extern "C" mako_status mako_pairs_class_flops(mako_pairs p, double thresh, int shard, int nshards, double* flops,
+                                              long long* quartets) {
+  try {
+    std::vector<double> fl;
+    std::vector<long long> nq, npq;
+    mako_status st = class_flops(p, thresh, shard, nshards, fl, nq, npq);
+    if (st) return st;
+    for (size_t i = 0; i < fl.size(); ++i) {
+      if (flops) flops[i] = fl[i];
+      if (quartets) quartets[i] = nq[i];
+    }
+    return MAKO_OK;
+  } catch (const std::exception& e) {
+    return fail(MAKO_ERR_OOM, e.what());
+  }
+}
+
+static void drop_events(mako_pairs p) {
+  for (auto& e : p->prof_events) {
+    cudaEventDestroy((cudaEvent_t)e.second.first);
+    cudaEventDestroy((cudaEvent_t)e.second.second);
+  }
+  p->prof_events.clear();
+}
+
+mako_pairs_s::~mako_pairs_s() { drop_events(this); }
+
+extern "C" mako_status mako_profile_enable(mako_pairs p, int enable) {
+  mako_status st;
+  if ((st = check_pairs(p))) return st;
+  drop_events(p);
+  p->prof = enable != 0;
+  return MAKO_OK;
+}
+
+extern "C" mako_status mako_profile_read(mako_pairs p, double* ms, long long* launches) {
+  mako_status st;
+  if ((st = check_pairs(p))) return st;
+  const int NC = NBUCKET * (NBUCKET + 1) / 2;
+  std::vector<double> t(NC, 0.0);
+  std::vector<long long> n(NC, 0);
+  for (auto& e : p->prof_events) {
+    cudaError_t ce = cudaEventSynchronize((cudaEvent_t)e.second.second);
+    if (ce != cudaSuccess) return cuda_check(ce, "cudaEventSynchronize");
+    float x = 0.f;
+    cudaEventElapsedTime(&x, (cudaEvent_t)e.second.first, (cudaEvent_t)e.second.second);
+    t[e.first] += x;
+    n[e.first] += 1;
+  }
+  for (int i = 0; i < NC; ++i) {
+    if (ms) ms[i] = t[i];
+    if (launches) launches[i] = n[i];
+  }
+  return MAKO_OK;
 }
 
 extern "C" mako_status mako_build_jk_launches(mako_pairs p, double thresh, int shard, int nshards, int* n) {
@@ -245,7 +318,7 @@ extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thres
       a.task_off = c.d_task_off.as<long long>();
       a.nket = c.d_nket.as<int>();
       a.nbra = (int)c.nket.size();
-      a.KT = p->plan.KT;
+      a.KT = c.KT;
       a.counter = p->d_counters.as<unsigned long long>() + class_index(c.X, c.Y);
       a.D = D;
       a.J = J;
@@ -254,7 +327,17 @@ extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thres
       a.ao = B->d_ao.as<int>();
       a.thresh = thresh;
       a.boys = B->d_boys.as<double>();
+      cudaEvent_t e0 = nullptr, e1 = nullptr;
+      if (p->prof) {
+        cudaEventCreate(&e0);
+        cudaEventCreate(&e1);
+        cudaEventRecord(e0, s);
+      }
       if ((st = launch_jk_class(c.X, c.Y, a, cuda_stream, &nl))) return st;
+      if (p->prof) {
+        cudaEventRecord(e1, s);
+        p->prof_events.push_back({class_index(c.X, c.Y), {(void*)e0, (void*)e1}});
+      }
     }
     symmetrize_kernel<<<592, 256, 0, s>>>(J, K, n);
     return cuda_check(cudaGetLastError(), "symmetrize launch");

@@ -43,6 +43,19 @@ constexpr int BOYS_MMAX = 24;         // supports L + 6 <= 24
 constexpr int BOYS_NM = BOYS_MMAX + 1;
 constexpr int BOYS_TAYLOR = 7;        // Taylor terms (|dT| <= 1/64 -> truncation < 5e-17 relative)
 
+// Kernel family per class (X >= Y buckets).  Low-l classes use the lane-per-ket register kernel
+// ("TPQ": Boys, R, contraction and digestion in registers of one lane), the rest the warp-per-quartet
+// DMMA kernel.  Register estimate (doubles): R + V + W + cached ket E~ + cached bra E~.
+MK_HD constexpr int b_la(int b) { return b >= 6 ? 3 : (b >= 3 ? 2 : (b >= 1 ? 1 : 0)); }
+MK_HD constexpr int b_lb(int b) { return b - b_la(b) * (b_la(b) + 1) / 2; }
+MK_HD constexpr int tpq_regs(int X, int Y) {
+  return nH(b_la(X) + b_lb(X) + b_la(Y) + b_lb(Y)) + nsph(b_la(X)) * nsph(b_lb(X)) * nsph(b_la(Y)) * nsph(b_lb(Y)) +
+         nsph(b_la(Y)) * nsph(b_lb(Y)) * (1 + nH(b_la(Y) + b_lb(Y))) +
+         (nsph(b_la(X)) * nsph(b_lb(X)) * nH(b_la(X) + b_lb(X)) <= 40 ? nsph(b_la(X)) * nsph(b_lb(X)) * nH(b_la(X) + b_lb(X)) : 0);
+}
+MK_HD constexpr bool use_tpq(int X, int Y) { return Y <= 1 && tpq_regs(X, Y) <= 100; }
+MK_HD constexpr int class_kt(int X, int Y) { return use_tpq(X, Y) ? 32 : 16; }
+
 // primitive-pair screening (reading R7)
 constexpr double PRIM_PAIR_EPS = 1e-18;
 

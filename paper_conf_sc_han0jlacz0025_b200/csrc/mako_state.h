@@ -55,6 +55,7 @@ struct PairSet {
 // per-class plan for one threshold
 struct ClassPlan {
   int X = 0, Y = 0;                // bra / ket buckets (X >= Y)
+  int KT = 16;                     // kets per task
   long long ntask = 0;             // tasks of the whole class (all shards)
   long long nquartet = 0;
   std::vector<int> nket;           // [nbra]
@@ -89,6 +90,10 @@ struct mako_pairs_s {
   mako::PairSet set;
   mako::Plan plan;
   mako::DevBuf d_counters;      // [55] task counters
+  // profiling (mako_profile_enable / read)
+  bool prof = false;
+  std::vector<std::pair<int, std::pair<void*, void*>>> prof_events;  // (class, (start, stop)) cudaEvent_t
+  ~mako_pairs_s();
 };
 
 namespace mako {

@@ -101,6 +101,24 @@ class Pairs:
                                                nshards, ctypes.byref(n)))
         return n.value
 
+    def class_flops(self, thresh=None, shard=0, nshards=1):
+        f = np.zeros(_lib.NCLASS)
+        q = np.zeros(_lib.NCLASS, np.int64)
+        check(self._lib.mako_pairs_class_flops(self.handle, float(self.tau if thresh is None else thresh), shard,
+                                               nshards, f.ctypes.data_as(ctypes.POINTER(ctypes.c_double)),
+                                               q.ctypes.data_as(ctypes.POINTER(ctypes.c_longlong))))
+        return f, q
+
+    def profile(self, enable=True):
+        check(self._lib.mako_profile_enable(self.handle, 1 if enable else 0))
+
+    def profile_read(self):
+        ms = np.zeros(_lib.NCLASS)
+        n = np.zeros(_lib.NCLASS, np.int64)
+        check(self._lib.mako_profile_read(self.handle, ms.ctypes.data_as(ctypes.POINTER(ctypes.c_double)),
+                                          n.ctypes.data_as(ctypes.POINTER(ctypes.c_longlong))))
+        return ms, n
+
     def close(self):
         if getattr(self, "handle", None):
             self._lib.mako_pairs_destroy(self.handle)

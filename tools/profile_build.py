@@ -1,0 +1,24 @@
+"""One J/K build of a config (for ncu captures): python tools/profile_build.py [--config X] [--builds N]"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import mako_inputs as mi  # noqa: E402
+from paper_conf_sc_han0jlacz0025_b200 import Basis, Pairs, build_jk  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="valinomycin-def2tzvp")
+ap.add_argument("--builds", type=int, default=1)
+ap.add_argument("--tau", type=float, default=1e-12)
+a = ap.parse_args()
+mol, basis = mi.config_molecule(a.config)
+sh = mi.shells_for(mol, basis)
+P = Pairs(Basis(mol.Z, mol.xyz_bohr, sh), a.tau)
+D = torch.tensor(mi.synthetic_density(sh.nbf(), mol.nelec // 2, seed=0), device="cuda")
+for _ in range(a.builds):
+    J, K = build_jk(P, D)
+torch.cuda.synchronize()
+print("done", float(J.abs().sum()), float(K.abs().sum()))
