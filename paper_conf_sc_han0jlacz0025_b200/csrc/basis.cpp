@@ -165,7 +165,7 @@ void boys_table(std::vector<double>& tab) {
   const int NP = 64, NG = 14;
   std::vector<long double> gx, gw;
   gauss_legendre(NG, gx, gw);
-  tab.assign((size_t)BOYS_NGRID * BOYS_NM, 0.0);
+  tab.assign(BOYS_TABLE_DOUBLES, 0.0);
   std::vector<long double> acc(BOYS_NM);
   for (int k = 0; k < BOYS_NGRID; ++k) {
     long double T = (long double)k * (long double)BOYS_H;
@@ -182,8 +182,11 @@ void boys_table(std::vector<double>& tab) {
         }
       }
     }
-    for (int m = 0; m < BOYS_NM; ++m) tab[(size_t)k * BOYS_NM + m] = (double)acc[m];
+    for (int m = 0; m < BOYS_NM; ++m) tab[(size_t)k * BOYS_STRIDE + m] = (double)acc[m];
+    tab[(size_t)k * BOYS_STRIDE + BOYS_ECOL] = (double)expl(-T);
   }
+  for (int k = 0; k < BOYS_NEXP; ++k)
+    tab[(size_t)BOYS_NGRID * BOYS_STRIDE + k] = (double)expl(-(40.0L + (long double)k * (long double)BOYS_H));
 }
 
 }  // namespace mako

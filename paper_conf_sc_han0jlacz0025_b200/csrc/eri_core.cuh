@@ -93,33 +93,65 @@ __device__ void init_tables(uint16_t* htab, uint32_t* rtab) {
   }
 }
 
-// Boys F_m(T), m = 0..L: 7-term Taylor expansion of F_L about the nearest grid point, then the
-// downward recursion F_m = (2T F_{m+1} + e^{-T})/(2m+1); for T >= 40 the erf closed form of F_0
-// (erfc(sqrt 40) < 1e-18) and the upward recursion.
+// 1/sqrt(x) for positive normal x: float seed + two Newton steps (no slow path)
+__device__ __forceinline__ double rsqrt_fast(double x) {
+  double y = (double)rsqrtf((float)x);
+  const double h = 0.5 * x;
+  y = y * fma(-h * y, y, 1.5);
+  y = y * fma(-h * y, y, 1.5);
+  return y;
+}
+
+// Boys F_m(T), m = 0..L (PAPER.md:L177 lookup-table evaluation; accuracy contract: reading R1).
+//  T < 40:  7-term Taylor expansion of F_L about the nearest grid point T_k = k/32 (|x| <= 1/64),
+//           exp(-T) = exp(-T_k) * sum_j x^j/j! from the same row, then the exact downward
+//           recursion F_m = (2T F_{m+1} + e^{-T}) / (2m+1).
+//  T >= 40: F_0 = (1/2) sqrt(pi/T) (erfc(sqrt 40) < 1e-18), upward F_{m+1} = ((2m+1)F_m - e^{-T})/(2T)
+//           with exp(-T) from a second 1/32 grid for T < 80 and dropped beyond (< 1e-18 relative).
 template <int L>
 __device__ __forceinline__ void boys_eval(double T, const double* __restrict__ tab, double (&F)[L + 1]) {
   if (T < BOYS_TMAX) {
     const int k = __double2int_rn(T * (1.0 / BOYS_H));
-    const double x = k * BOYS_H - T;
-    const double* r = tab + k * BOYS_NM + L;
+    const double x = fma((double)k, BOYS_H, -T);
+    const double* r = tab + k * BOYS_STRIDE + L;
+    const double x2 = x * 0.5, x3 = x * (1.0 / 3.0), x4 = x * 0.25, x5 = x * 0.2, x6 = x * (1.0 / 6.0);
     double f = __ldg(r + 6);
-    f = fma(f, x * (1.0 / 6.0), __ldg(r + 5));
-    f = fma(f, x * (1.0 / 5.0), __ldg(r + 4));
-    f = fma(f, x * 0.25, __ldg(r + 3));
-    f = fma(f, x * (1.0 / 3.0), __ldg(r + 2));
-    f = fma(f, x * 0.5, __ldg(r + 1));
+    f = fma(f, x6, __ldg(r + 5));
+    f = fma(f, x5, __ldg(r + 4));
+    f = fma(f, x4, __ldg(r + 3));
+    f = fma(f, x3, __ldg(r + 2));
+    f = fma(f, x2, __ldg(r + 1));
     f = fma(f, x, __ldg(r));
     F[L] = f;
     if constexpr (L > 0) {
-      const double e = exp(-T), t2 = 2.0 * T;
+      double e = fma(x6, 1.0, 1.0);
+      e = fma(e, x5, 1.0);
+      e = fma(e, x4, 1.0);
+      e = fma(e, x3, 1.0);
+      e = fma(e, x2, 1.0);
+      e = fma(e, x, 1.0);
+      e *= __ldg(tab + k * BOYS_STRIDE + BOYS_ECOL);
+      const double t2 = 2.0 * T;
 #pragma unroll
       for (int m = L - 1; m >= 0; --m) F[m] = fma(t2, F[m + 1], e) * (1.0 / (2 * m + 1));
     }
   } else {
-    const double it = 1.0 / T;
-    F[0] = 0.5 * sqrt(PI_D * it);
+    const double rs = rsqrt_fast(T);
+    F[0] = 0.88622692545275801365 * rs;  // sqrt(pi)/2
     if constexpr (L > 0) {
-      const double e = exp(-T), h = 0.5 * it;
+      double e = 0.0;
+      if (T < BOYS_TEXP) {
+        const int k = __double2int_rn((T - BOYS_TMAX) * (1.0 / BOYS_H));
+        const double x = fma((double)k, BOYS_H, BOYS_TMAX - T);
+        double s = fma(x, 1.0 / 6.0, 1.0);
+        s = fma(s, x * 0.2, 1.0);
+        s = fma(s, x * 0.25, 1.0);
+        s = fma(s, x * (1.0 / 3.0), 1.0);
+        s = fma(s, x * 0.5, 1.0);
+        s = fma(s, x, 1.0);
+        e = s * __ldg(tab + (size_t)BOYS_NGRID * BOYS_STRIDE + k);
+      }
+      const double h = 0.5 * rs * rs;
 #pragma unroll
       for (int m = 0; m < L; ++m) F[m + 1] = fma((double)(2 * m + 1), F[m], -e) * h;
     }
@@ -135,12 +167,12 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
                                           double Qz, double* __restrict__ buf, const uint32_t* __restrict__ rtab,
                                           const double* __restrict__ btab, int lane) {
   constexpr int L = C::L, NH = C::NH;
-  const double pq = p + q, rho = p * q / pq;
+  const double pq = p + q, ri = rsqrt_fast(pq), rho = p * q * ri * ri;
   const double X = Px - Qx, Y = Py - Qy, Z = Pz - Qz;
   const double T = rho * (X * X + Y * Y + Z * Z);
   double F[L + 1];
   boys_eval<L>(T, btab, F);
-  double s = TWO_PI_52 / sqrt(pq);
+  double s = TWO_PI_52 * ri;
   const double m2r = -2.0 * rho;
 #pragma unroll
   for (int n = 0; n <= L; ++n) {

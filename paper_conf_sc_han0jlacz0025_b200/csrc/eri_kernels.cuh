@@ -45,18 +45,15 @@ __global__ void __launch_bounds__(CTA_THREADS) jk_kernel(JKArgs a) {
   double* V = Rbuf + C::W_R;
   double* jab = V + C::W_V;
   for (;;) {
-    unsigned long long tk = 0;
-    if (lane == 0) tk = atomicAdd(a.counter, 1ull);
-    tk = __shfl_sync(0xffffffffu, tk, 0);
-    const long long task = a.task_begin + (long long)tk;
-    if (task >= a.task_end) break;
-    // bra = largest P with task_off[P] <= task
-    int lo = 0, hi = a.nbra - 1;
-    while (lo < hi) {
-      const int mid = (lo + hi + 1) >> 1;
-      if (__ldg(a.task_off + mid) <= task) lo = mid; else hi = mid - 1;
-    }
-    const int P = lo;
+  unsigned long long grab = 0;
+  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
+  grab = __shfl_sync(0xffffffffu, grab, 0);
+  const long long tg0 = a.task_begin + (long long)grab;
+  if (tg0 >= a.task_end) break;
+  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  int P = find_bra(a.task_off, a.nbra, tg0);
+  for (long long task = tg0; task < tg1; ++task) {
+    while (__ldg(a.task_off + P + 1) <= task) ++P;
     const int r0 = (int)(task - __ldg(a.task_off + P)) * a.KT;
     const int r1 = min(r0 + a.KT, __ldg(a.nket + P));
     const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
@@ -78,6 +75,7 @@ __global__ void __launch_bounds__(CTA_THREADS) jk_kernel(JKArgs a) {
     for (int ab = lane; ab < C::NAB; ab += 32)
       atomicAdd(a.J + (size_t)(oa + ab / C::NB) * a.nbf + ob + ab % C::NB, jab[ab]);
     __syncwarp();
+  }
   }
 }
 

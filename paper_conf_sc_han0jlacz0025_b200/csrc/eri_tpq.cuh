@@ -74,11 +74,11 @@ __device__ __forceinline__ void r_levels(double* R, const double* F, double X, d
 template <int L>
 __device__ __forceinline__ void r_regs(double p, double Px, double Py, double Pz, double q, double Qx, double Qy,
                                        double Qz, const double* __restrict__ btab, double (&R)[nH(L)]) {
-  const double pq = p + q, rho = p * q / pq;
+  const double pq = p + q, ri = rsqrt_fast(pq), rho = p * q * ri * ri;
   const double X = Px - Qx, Y = Py - Qy, Z = Pz - Qz;
   double F[L + 1];
   boys_eval<L>(rho * (X * X + Y * Y + Z * Z), btab, F);
-  double s = TWO_PI_52 * rsqrt(pq);
+  double s = TWO_PI_52 * ri;
   const double m2r = -2.0 * rho;
 #pragma unroll
   for (int n = 0; n <= L; ++n) {
@@ -89,25 +89,41 @@ __device__ __forceinline__ void r_regs(double p, double Px, double Py, double Pz
   r_levels<L, L - 1>(R, F, X, Y, Z);
 }
 
+// W-accumulation variant fits in registers (R + V + W + ket E~, doubles)?
+template <class C>
+constexpr bool tpq_wacc() {
+  return nH(C::L) + C::NAB * C::NCD + C::NHAB * C::NCD + C::NHCD * C::NCD <= 110;
+}
+
+constexpr int TASK_GRAB = 4;  // tasks taken per counter increment (one bra search per grab)
+
+__device__ __forceinline__ int find_bra(const long long* __restrict__ task_off, int nbra, long long task) {
+  int lo = 0, hi = nbra - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (__ldg(task_off + mid) <= task) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
 // Persistent lane-per-ket kernel (JKArgs.KT must be 32).
 template <int X, int Y>
 __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
   using C = ClsXY<X, Y>;
   constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
   constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND;
+  constexpr bool WACC = tpq_wacc<C>();
   const int lane = threadIdx.x & 31;
   for (;;) {
-    unsigned long long tk = 0;
-    if (lane == 0) tk = atomicAdd(a.counter, 1ull);
-    tk = __shfl_sync(0xffffffffu, tk, 0);
-    const long long task = a.task_begin + (long long)tk;
-    if (task >= a.task_end) break;
-    int lo = 0, hi = a.nbra - 1;
-    while (lo < hi) {
-      const int mid = (lo + hi + 1) >> 1;
-      if (__ldg(a.task_off + mid) <= task) lo = mid; else hi = mid - 1;
-    }
-    const int P = lo;
+  unsigned long long grab = 0;
+  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
+  grab = __shfl_sync(0xffffffffu, grab, 0);
+  const long long tg0 = a.task_begin + (long long)grab;
+  if (tg0 >= a.task_end) break;
+  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  int P = find_bra(a.task_off, a.nbra, tg0);
+  for (long long task = tg0; task < tg1; ++task) {
+    while (__ldg(a.task_off + P + 1) <= task) ++P;
     const int r0 = (int)(task - __ldg(a.task_off + P)) * 32;
     const int r1 = min(r0 + 32, __ldg(a.nket + P));
     const int R = r0 + lane;
@@ -126,6 +142,48 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
       sc = __ldg(a.ket.shA + R);
       sd = __ldg(a.ket.shB + R);
       const int k0 = __ldg(a.ket.poff + R), k1 = __ldg(a.ket.poff + R + 1);
+      if constexpr (WACC) {
+        // bra primitive outer: W[p][cd] = sum_kl sum_q R_{p+q} E~_cd[q][cd], then V += E~_ab W
+        for (int ij = b0; ij < b1; ++ij) {
+          const double p = __ldg(a.bra.pdat + 4 * ij), Px = __ldg(a.bra.pdat + 4 * ij + 1),
+                       Py = __ldg(a.bra.pdat + 4 * ij + 2), Pz = __ldg(a.bra.pdat + 4 * ij + 3);
+          double W[NHAB][NCD];
+#pragma unroll
+          for (int h = 0; h < NHAB; ++h)
+#pragma unroll
+            for (int j = 0; j < NCD; ++j) W[h][j] = 0.0;
+          for (int kl = k0; kl < k1; ++kl) {
+            const double q = __ldg(a.ket.pdat + 4 * kl), Qx = __ldg(a.ket.pdat + 4 * kl + 1),
+                         Qy = __ldg(a.ket.pdat + 4 * kl + 2), Qz = __ldg(a.ket.pdat + 4 * kl + 3);
+            double Ek[NHCD][NCD];
+            const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
+#pragma unroll
+            for (int h = 0; h < NHCD; ++h)
+#pragma unroll
+              for (int j = 0; j < NCD; ++j) Ek[h][j] = __ldg(ek + h * NCD + j);
+            double Rr[nH(L)];
+            r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
+            static_for<0, NHAB>([&](auto pc) {
+              constexpr int pp = decltype(pc)::value;
+              static_for<0, NHCD>([&](auto qc) {
+                constexpr int qq = decltype(qc)::value;
+                constexpr int hs = h_sum(pp, qq);
+#pragma unroll
+                for (int j = 0; j < NCD; ++j) W[pp][j] = fma(Rr[hs], Ek[qq][j], W[pp][j]);
+              });
+            });
+          }
+          const double* __restrict__ eb = a.bra.Ebra + (size_t)ij * (NAB * NHAB);
+#pragma unroll
+          for (int i = 0; i < NAB; ++i)
+#pragma unroll
+            for (int h = 0; h < NHAB; ++h) {
+              const double e = __ldg(eb + i * NHAB + h);
+#pragma unroll
+              for (int j = 0; j < NCD; ++j) V[i][j] = fma(e, W[h][j], V[i][j]);
+            }
+        }
+      } else {
       for (int kl = k0; kl < k1; ++kl) {
         const double q = __ldg(a.ket.pdat + 4 * kl), Qx = __ldg(a.ket.pdat + 4 * kl + 1),
                      Qy = __ldg(a.ket.pdat + 4 * kl + 2), Qz = __ldg(a.ket.pdat + 4 * kl + 3);
@@ -161,6 +219,7 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
             }
           });
         }
+      }
       }
     }
     // ---- digestion (a9) ----
@@ -245,6 +304,7 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
           for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (oa + i) * n + oc + k), s);
         atomicAdd(a.K + (ob + j) * n + od + l, deg * s);
       }
+  }
   }
 }
 
