@@ -356,7 +356,8 @@ def run_mako(args):
     if args.class_times and rank == 0:
         line["class_ms"] = {f"({names[int((math.isqrt(8*i+1)-1)//2)]}|"
                             f"{names[i - int((math.isqrt(8*i+1)-1)//2) * (int((math.isqrt(8*i+1)-1)//2) + 1) // 2]})":
-                            [round(float(cls_ms[i] / max(cls_n[i], 1)), 4), float(cls_flops[i]), int(cls_q[i])]
+                            [round(float(cls_ms[i] / max(cls_n[i], 1)), 4), float(cls_flops[i]), int(cls_q[i]),
+                             int(P.last_prim_quartets[i])]
                             for i in range(len(cls_ms)) if cls_n[i] > 0}
     if rank == 0:
         print(json.dumps(line), flush=True)

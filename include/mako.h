@@ -123,9 +123,9 @@ mako_status mako_build_jk_launches(mako_pairs pairs, double thresh, int shard, i
 #define MAKO_NCLASS 55
 
 /* Per-class algorithmic GEMM FLOPs (same definition as mako_pairs_flops) and quartet counts of
- * shard `shard`/`nshards` at thresh.  flops[MAKO_NCLASS], quartets[MAKO_NCLASS] (HOST, either NULL). */
+ * shard `shard`/`nshards` at thresh.  flops, quartets, prim_quartets: HOST arrays of MAKO_NCLASS (any NULL). */
 mako_status mako_pairs_class_flops(mako_pairs pairs, double thresh, int shard, int nshards, double* flops,
-                                   long long* quartets);
+                                   long long* quartets, long long* prim_quartets);
 
 /* Measurement hooks.  mako_profile_enable(pairs, 1) resets and starts recording a CUDA event pair
  * around every class-kernel launch of subsequent mako_build_jk calls (on their stream);

@@ -59,8 +59,8 @@ def load():
         "mako_build_jk_launches": ([_vp, ctypes.c_double, ctypes.c_int, ctypes.c_int, _ip], ctypes.c_int),
         "mako_eri_batch": ([_vp, ctypes.c_int, _ip, _vp, ctypes.c_size_t, _vp], ctypes.c_int),
         "mako_boys": ([ctypes.c_int, _vp, ctypes.c_int, _vp, _vp], ctypes.c_int),
-        "mako_pairs_class_flops": ([_vp, ctypes.c_double, ctypes.c_int, ctypes.c_int, _dp, ctypes.POINTER(_ll)],
-                                   ctypes.c_int),
+        "mako_pairs_class_flops": ([_vp, ctypes.c_double, ctypes.c_int, ctypes.c_int, _dp, ctypes.POINTER(_ll),
+                                    ctypes.POINTER(_ll)], ctypes.c_int),
         "mako_profile_enable": ([_vp, ctypes.c_int], ctypes.c_int),
         "mako_profile_read": ([_vp, _dp, ctypes.POINTER(_ll)], ctypes.c_int),
         "mako_last_error": ([], ctypes.c_char_p),

@@ -22,6 +22,7 @@ int jk_blocks_per_sm();
 #ifdef MAKO_DEFINE_KERNELS
 #include "eri_core.cuh"
 #include "eri_tpq.cuh"
+#include "eri_slab.cuh"
 
 namespace mako {
 
@@ -144,6 +145,10 @@ int jk_blocks_per_sm() {
     int nb = 0;
     if constexpr (use_tpq(X, Y)) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, tpq_jk_kernel<X, Y>, CTA_THREADS, 0);
+    } else if constexpr (use_slab<X, Y>()) {
+      constexpr size_t ss = SlabCfg<X, Y>::SMEM;
+      if (set_smem_attr<X, Y>((const void*)slab_jk_kernel<X, Y>, ss)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, slab_jk_kernel<X, Y>, CTA_THREADS, ss);
     } else {
       if (set_smem_attr<X, Y>((const void*)jk_kernel<X, Y>, smem)) return 1;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel<X, Y>, CTA_THREADS, smem);
@@ -168,6 +173,8 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   const int grid = (int)(want < cap ? want : cap);
   if constexpr (use_tpq(X, Y))
     tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, (cudaStream_t)stream>>>(a);
+  else if constexpr (use_slab<X, Y>())
+    slab_jk_kernel<X, Y><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
   else
     jk_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
   cudaError_t e = cudaGetLastError();

@@ -218,7 +218,7 @@ extern "C" mako_status mako_pairs_flops(mako_pairs p, double thresh, int shard, 
 }
 
 extern "C" mako_status mako_pairs_class_flops(mako_pairs p, double thresh, int shard, int nshards, double* flops,
-                                              long long* quartets) {
+                                              long long* quartets, long long* prim_quartets) {
   try {
     std::vector<double> fl;
     std::vector<long long> nq, npq;
@@ -227,6 +227,7 @@ extern "C" mako_status mako_pairs_class_flops(mako_pairs p, double thresh, int s
     for (size_t i = 0; i < fl.size(); ++i) {
       if (flops) flops[i] = fl[i];
       if (quartets) quartets[i] = nq[i];
+      if (prim_quartets) prim_quartets[i] = npq[i];
     }
     return MAKO_OK;
   } catch (const std::exception& e) {

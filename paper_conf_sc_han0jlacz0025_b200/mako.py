@@ -104,9 +104,12 @@ class Pairs:
     def class_flops(self, thresh=None, shard=0, nshards=1):
         f = np.zeros(_lib.NCLASS)
         q = np.zeros(_lib.NCLASS, np.int64)
+        pq = np.zeros(_lib.NCLASS, np.int64)
+        llp = lambda x: x.ctypes.data_as(ctypes.POINTER(ctypes.c_longlong))
         check(self._lib.mako_pairs_class_flops(self.handle, float(self.tau if thresh is None else thresh), shard,
-                                               nshards, f.ctypes.data_as(ctypes.POINTER(ctypes.c_double)),
-                                               q.ctypes.data_as(ctypes.POINTER(ctypes.c_longlong))))
+                                               nshards, f.ctypes.data_as(ctypes.POINTER(ctypes.c_double)), llp(q),
+                                               llp(pq)))
+        self.last_prim_quartets = pq
         return f, q
 
     def profile(self, enable=True):

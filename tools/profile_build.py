@@ -13,12 +13,14 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="valinomycin-def2tzvp")
 ap.add_argument("--builds", type=int, default=1)
 ap.add_argument("--tau", type=float, default=1e-12)
+ap.add_argument("--shard", type=int, default=0)
+ap.add_argument("--nshards", type=int, default=1)
 a = ap.parse_args()
 mol, basis = mi.config_molecule(a.config)
 sh = mi.shells_for(mol, basis)
 P = Pairs(Basis(mol.Z, mol.xyz_bohr, sh), a.tau)
 D = torch.tensor(mi.synthetic_density(sh.nbf(), mol.nelec // 2, seed=0), device="cuda")
 for _ in range(a.builds):
-    J, K = build_jk(P, D)
+    J, K = build_jk(P, D, shard=a.shard, nshards=a.nshards)
 torch.cuda.synchronize()
 print("done", float(J.abs().sum()), float(K.abs().sum()))
