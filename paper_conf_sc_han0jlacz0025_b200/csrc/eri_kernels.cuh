@@ -16,6 +16,8 @@ template <int X, int Y>
 mako_status launch_batch_xy(const BatchArgs& a, void* stream);
 template <int X, int Y>
 int jk_blocks_per_sm();
+template <int X, int Y>
+int task_kets_xy();
 
 }  // namespace mako
 
@@ -23,6 +25,7 @@ int jk_blocks_per_sm();
 #include "eri_core.cuh"
 #include "eri_tpq.cuh"
 #include "eri_slab.cuh"
+#include "eri_kf.cuh"
 
 namespace mako {
 
@@ -52,11 +55,12 @@ __global__ void __launch_bounds__(CTA_THREADS) jk_kernel(JKArgs a) {
   const long long tg0 = a.task_begin + (long long)grab;
   if (tg0 >= a.task_end) break;
   const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
-  int P = find_bra(a.task_off, a.nbra, tg0);
+  int U = find_bra(a.task_off, a.nbra, tg0);
   for (long long task = tg0; task < tg1; ++task) {
-    while (__ldg(a.task_off + P + 1) <= task) ++P;
-    const int r0 = (int)(task - __ldg(a.task_off + P)) * a.KT;
-    const int r1 = min(r0 + a.KT, __ldg(a.nket + P));
+    while (__ldg(a.task_off + U + 1) <= task) ++U;
+    const int P = U / a.ngroup;  // flat index = bra pair x ket primitive-count group
+    const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * a.KT;
+    const int r1 = min(r0 + a.KT, __ldg(a.kend + U));
     const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
     const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
     const double QP = __ldg(a.bra.Q + P);
@@ -143,7 +147,11 @@ int jk_blocks_per_sm() {
   static int cached = -1;
   if (cached < 0) {
     int nb = 0;
-    if constexpr (use_tpq(X, Y)) {
+    if constexpr (use_kf<X, Y>()) {
+      constexpr size_t ks = KfCfg<X, Y>::SMEM;
+      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel<X, Y>, ks)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel<X, Y>, CTA_THREADS, ks);
+    } else if constexpr (use_tpq(X, Y)) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, tpq_jk_kernel<X, Y>, CTA_THREADS, 0);
     } else if constexpr (use_slab<X, Y>()) {
       constexpr size_t ss = SlabCfg<X, Y>::SMEM;
@@ -171,7 +179,9 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   long long want = (ntask + CTA_WARPS - 1) / CTA_WARPS;
   long long cap = (long long)nsm * bps;
   const int grid = (int)(want < cap ? want : cap);
-  if constexpr (use_tpq(X, Y))
+  if constexpr (use_kf<X, Y>())
+    kf_jk_kernel<X, Y><<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
+  else if constexpr (use_tpq(X, Y))
     tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, (cudaStream_t)stream>>>(a);
   else if constexpr (use_slab<X, Y>())
     slab_jk_kernel<X, Y><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
@@ -200,8 +210,18 @@ mako_status launch_batch_xy(const BatchArgs& a, void* stream) {
 
 }  // namespace mako
 
+namespace mako {
+template <int X, int Y>
+int task_kets_xy() {
+  if constexpr (use_kf<X, Y>()) return KfCfg<X, Y>::NK;
+  else if constexpr (use_tpq(X, Y)) return 32;
+  else return 16;
+}
+}  // namespace mako
+
 #define MAKO_INSTANTIATE(X, Y)                                                                   \
   template mako_status mako::launch_jk_xy<X, Y>(const mako::JKArgs&, void*, int*);               \
   template mako_status mako::launch_batch_xy<X, Y>(const mako::BatchArgs&, void*);               \
-  template int mako::jk_blocks_per_sm<X, Y>();
+  template int mako::jk_blocks_per_sm<X, Y>();                                                   \
+  template int mako::task_kets_xy<X, Y>();
 #endif

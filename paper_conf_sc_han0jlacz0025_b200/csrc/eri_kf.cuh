@@ -1,0 +1,232 @@
+// eri_kf.cuh -- "ket-first" kernel for classes with a light ket (ss, ps, pp, ds) and a heavier bra.
+//
+// Eq. 7 evaluated in the cheaper order for n_cd << n_ab, with the two stages on
+// the two separate FP64 pipes of sm_100a (S6: DFMA and DMMA run concurrently):
+//   DFMA (per lane, registers):  W^{ij}[p][cd] = sum_kl sum_q R^{(ij,kl)}_{p+q} (-1)^{|q|} E~_cd^{kl}[q][cd]
+//                                (Boys a4 + Eq. 5 a5 + the ket contraction, a striped layout: lanes own kets)
+//   DMMA (warp, mma.sync f64):   V[ab][(k,cd)] += sum_p E~_ab^{ij}[ab][p] W^{ij}[p][(k,cd)]
+//                                (the bra contraction as one GEMM with N = kets x cd; the blocked layout of
+//                                L233-L249 is the SMEM hand-off of W)
+// A warp owns one bra pair and NK kets; 32/NK lanes share a ket and split its p range (each lane
+// recomputes the ket's R -- cheaper than synchronising).  Digestion (a9) is spread over the lanes of
+// each ket; J_ab is reduced across kets with warp shuffles.
+#pragma once
+
+#include "eri_core.cuh"
+#include "eri_tpq.cuh"
+
+namespace mako {
+
+template <int X, int Y>
+struct KfCfg {
+  using C = ClsXY<X, Y>;
+  static constexpr int vfr(int nk) { return C::MT * ((nk * C::NCD + 7) / 8) * 2; }
+  static constexpr int wpart(int nk) { return ((C::NHAB + (32 / nk) - 1) / (32 / nk)) * C::NCD; }
+  static constexpr int regs(int nk) { return nH(C::L) + wpart(nk) + vfr(nk); }
+  static constexpr int pick() {
+    return (vfr(16) <= 24 && regs(16) <= 128) ? 16
+                                              : ((vfr(8) <= 24 && regs(8) <= 128) ? 8
+                                                                                  : ((vfr(4) <= 24 && regs(4) <= 128) ? 4 : 0));
+  }
+  static constexpr int NK = pick();                      // kets per warp task
+  static constexpr int LPK = NK ? 32 / NK : 1;           // lanes per ket
+  static constexpr int PP = (C::NHAB + LPK - 1) / LPK;   // p values per lane
+  static constexpr int NTV = (NK * C::NCD + 7) / 8;      // n8 tiles of V / W columns
+  static constexpr int COLS = NTV * 8;
+  static constexpr int WS = COLS + ((4 - COLS % 16) + 16) % 16;  // row stride = 4 (mod 16): conflict-free B loads
+  static constexpr int ROWS = (C::MT * 8 > C::KS1 * 4) ? C::MT * 8 : C::KS1 * 4;
+  static constexpr int WARP_DBL = ROWS * WS;
+  static constexpr size_t SMEM = sizeof(double) * 4 * WARP_DBL;
+  static constexpr bool OK = NK > 0 && Y <= 3 && C::L <= 6;
+};
+
+template <int X, int Y>
+constexpr bool use_kf() {
+  // measured per class on the valinomycin-sized workload (profiles/README.md): KF wins for light kets
+  // with a heavier bra; pp kets (8-fold redundant R per ket) stay on the slot-batched kernel
+  constexpr int c = X * 100 + Y;
+  constexpr bool pick = c == 303 || c == 401 || c == 403 || c == 501 || c == 603 || c == 701 || c == 800 ||
+                        c == 801 || c == 900 || c == 700 || c == 500;
+  return KfCfg<X, Y>::OK && pick;
+}
+
+template <int X, int Y>
+__global__ void __launch_bounds__(128) kf_jk_kernel(JKArgs a) {
+  using C = ClsXY<X, Y>;
+  using K = KfCfg<X, Y>;
+  constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
+  constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND;
+  constexpr int MT = C::MT, KS1 = C::KS1, NK = K::NK, LPK = K::LPK, PP = K::PP, NTV = K::NTV, WS = K::WS;
+  extern __shared__ __align__(16) double kf_smem[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int g = lane >> 2, t = lane & 3;
+  const int kk = lane / LPK, hh = lane % LPK;
+  double* Ws = kf_smem + (size_t)warp * K::WARP_DBL;
+  for (int i = lane; i < K::WARP_DBL; i += 32) Ws[i] = 0.0;  // padding rows/cols stay zero forever
+  __syncwarp();
+  for (;;) {
+  unsigned long long grab = 0;
+  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
+  grab = __shfl_sync(0xffffffffu, grab, 0);
+  const long long tg0 = a.task_begin + (long long)grab;
+  if (tg0 >= a.task_end) break;
+  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  int U = find_bra(a.task_off, a.nbra, tg0);
+  for (long long task = tg0; task < tg1; ++task) {
+    while (__ldg(a.task_off + U + 1) <= task) ++U;
+    const int P = U / a.ngroup;  // flat index = bra pair x ket primitive-count group
+    const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * NK;
+    const int r1 = min(r0 + NK, __ldg(a.kend + U));
+    const int R = r0 + kk;
+    const double QP = __ldg(a.bra.Q + P);
+    const bool active = R < r1 && QP * __ldg(a.ket.Q + min(R, r1 - 1)) >= a.thresh;
+    const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
+    const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
+    const int b0 = __ldg(a.bra.poff + P), b1 = __ldg(a.bra.poff + P + 1);
+    const int k0 = active ? __ldg(a.ket.poff + R) : 0, k1 = active ? __ldg(a.ket.poff + R + 1) : 0;
+    double vf[MT][NTV][2];
+#pragma unroll
+    for (int m = 0; m < MT; ++m)
+#pragma unroll
+      for (int n = 0; n < NTV; ++n) vf[m][n][0] = vf[m][n][1] = 0.0;
+    for (int ij = b0; ij < b1; ++ij) {
+      // ---- DFMA stage: this lane's p-slice of W^{ij} for its ket ----
+      const double p = __ldg(a.bra.pdat + 4 * ij), Px = __ldg(a.bra.pdat + 4 * ij + 1),
+                   Py = __ldg(a.bra.pdat + 4 * ij + 2), Pz = __ldg(a.bra.pdat + 4 * ij + 3);
+      double W[PP][NCD];
+#pragma unroll
+      for (int i = 0; i < PP; ++i)
+#pragma unroll
+        for (int j = 0; j < NCD; ++j) W[i][j] = 0.0;
+      for (int kl = k0; kl < k1; ++kl) {
+        const double q = __ldg(a.ket.pdat + 4 * kl), Qx = __ldg(a.ket.pdat + 4 * kl + 1),
+                     Qy = __ldg(a.ket.pdat + 4 * kl + 2), Qz = __ldg(a.ket.pdat + 4 * kl + 3);
+        double Rr[nH(L)];
+        r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
+        const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
+        static_for<0, LPK>([&](auto hc) {
+          constexpr int H = decltype(hc)::value;
+          constexpr int p0 = H * PP, p1 = (p0 + PP < NHAB) ? p0 + PP : NHAB;
+          if (hh == H) {
+            static_for<0, NHCD>([&](auto qc) {
+              constexpr int qq = decltype(qc)::value;
+              double e[NCD];
+#pragma unroll
+              for (int j = 0; j < NCD; ++j) e[j] = __ldg(ek + qq * NCD + j);
+              static_for<p0, p1>([&](auto pc) {
+                constexpr int pp = decltype(pc)::value;
+                constexpr int hs = h_sum(pp, qq);
+#pragma unroll
+                for (int j = 0; j < NCD; ++j) W[pp - p0][j] = fma(Rr[hs], e[j], W[pp - p0][j]);
+              });
+            });
+          }
+        });
+      }
+      // SL -> BL hand-off: W slice to SMEM row p, column (ket, cd)
+#pragma unroll
+      for (int i = 0; i < PP; ++i) {
+        const int pr = hh * PP + i;
+        if (pr < NHAB)
+#pragma unroll
+          for (int j = 0; j < NCD; ++j) Ws[pr * WS + kk * NCD + j] = W[i][j];
+      }
+      __syncwarp();
+      // ---- DMMA stage: V[ab][(k,cd)] += E~_ab^{ij} W ----
+      const double* __restrict__ E = a.bra.Ebra + (size_t)ij * (NAB * NHAB);
+#pragma unroll
+      for (int ks = 0; ks < KS1; ++ks) {
+        const int pc = 4 * ks + t;
+        double af[MT];
+#pragma unroll
+        for (int m = 0; m < MT; ++m) {
+          const int row = 8 * m + g;
+          af[m] = (row < NAB && pc < NHAB) ? __ldg(E + row * NHAB + pc) : 0.0;
+        }
+#pragma unroll
+        for (int n = 0; n < NTV; ++n) {
+          const double b = Ws[pc * WS + 8 * n + g];
+#pragma unroll
+          for (int m = 0; m < MT; ++m) dmma884(vf[m][n][0], vf[m][n][1], af[m], b);
+        }
+      }
+      __syncwarp();
+    }
+    // ---- V fragments to SMEM (rows ab, columns (k, cd)) ----
+#pragma unroll
+    for (int m = 0; m < MT; ++m)
+#pragma unroll
+      for (int n = 0; n < NTV; ++n)
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int row = 8 * m + g, col = 8 * n + 2 * t + i;
+          if (row < NAB && col < NK * NCD) Ws[row * WS + col] = vf[m][n][i];
+        }
+    __syncwarp();
+    // ---- digestion (a9) ----
+    const int sc = active ? __ldg(a.ket.shA + R) : 0, sd = active ? __ldg(a.ket.shB + R) : 0;
+    double deg = 1.0;
+    if (sa == sb) deg *= 0.5;
+    if (sc == sd) deg *= 0.5;
+    if (a.same_bucket && P == R) deg *= 0.5;
+    if (!active) deg = 0.0;
+    const int oc = active ? __ldg(a.ao + sc) : 0, od = active ? __ldg(a.ao + sd) : 0;
+    const double* __restrict__ Dm = a.D;
+    const size_t nb = (size_t)a.nbf;
+    const double* Vk = Ws + kk * NCD;  // V[ab][cd] of my ket = Vk[ab * WS + cd]
+    // J_ab: lanes with the same hh share ab; reduce over the kets
+    for (int i0 = 0; i0 < NAB; i0 += LPK) {
+      const int ab = i0 + hh;
+      double s = 0.0;
+      if (active && ab < NAB) {
+#pragma unroll
+        for (int k = 0; k < NC; ++k)
+#pragma unroll
+          for (int l = 0; l < ND; ++l) s = fma(Vk[ab * WS + k * ND + l], __ldg(Dm + (oc + k) * nb + od + l), s);
+      }
+      s *= deg;
+#pragma unroll
+      for (int o = LPK; o < 32; o <<= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+      if (kk == 0 && ab < NAB) atomicAdd(a.J + (oa + ab / NB) * nb + ob + ab % NB, 2.0 * s);
+    }
+    if (active) {
+      // J_cd
+      for (int cd = hh; cd < NCD; cd += LPK) {
+        double s = 0.0;
+        for (int i = 0; i < NA; ++i)
+          for (int j = 0; j < NB; ++j) s = fma(Vk[(i * NB + j) * WS + cd], __ldg(Dm + (oa + i) * nb + ob + j), s);
+        atomicAdd(a.J + (oc + cd / ND) * nb + od + cd % ND, 2.0 * deg * s);
+      }
+      // K_ac (NA*NC) | K_ad (NA*ND) | K_bc (NB*NC) | K_bd (NB*ND), flattened over the lanes of the ket
+      constexpr int N1 = NA * NC, N2 = N1 + NA * ND, N3 = N2 + NB * NC, N4 = N3 + NB * ND;
+      for (int x = hh; x < N4; x += LPK) {
+        double s = 0.0;
+        if (x < N1) {
+          const int i = x / NC, k = x % NC;
+          for (int j = 0; j < NB; ++j)
+            for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (ob + j) * nb + od + l), s);
+          atomicAdd(a.K + (oa + i) * nb + oc + k, deg * s);
+        } else if (x < N2) {
+          const int y = x - N1, i = y / ND, l = y % ND;
+          for (int j = 0; j < NB; ++j)
+            for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (ob + j) * nb + oc + k), s);
+          atomicAdd(a.K + (oa + i) * nb + od + l, deg * s);
+        } else if (x < N3) {
+          const int y = x - N2, j = y / NC, k = y % NC;
+          for (int i = 0; i < NA; ++i)
+            for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (oa + i) * nb + od + l), s);
+          atomicAdd(a.K + (ob + j) * nb + oc + k, deg * s);
+        } else {
+          const int y = x - N3, j = y / ND, l = y % ND;
+          for (int i = 0; i < NA; ++i)
+            for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (oa + i) * nb + oc + k), s);
+          atomicAdd(a.K + (ob + j) * nb + od + l, deg * s);
+        }
+      }
+    }
+    __syncwarp();
+  }
+  }
+}
+
+}  // namespace mako

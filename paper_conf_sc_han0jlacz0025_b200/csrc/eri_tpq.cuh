@@ -121,11 +121,12 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
   const long long tg0 = a.task_begin + (long long)grab;
   if (tg0 >= a.task_end) break;
   const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
-  int P = find_bra(a.task_off, a.nbra, tg0);
+  int U = find_bra(a.task_off, a.nbra, tg0);
   for (long long task = tg0; task < tg1; ++task) {
-    while (__ldg(a.task_off + P + 1) <= task) ++P;
-    const int r0 = (int)(task - __ldg(a.task_off + P)) * 32;
-    const int r1 = min(r0 + 32, __ldg(a.nket + P));
+    while (__ldg(a.task_off + U + 1) <= task) ++U;
+    const int P = U / a.ngroup;  // flat index = bra pair x ket primitive-count group
+    const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * 32;
+    const int r1 = min(r0 + 32, __ldg(a.kend + U));
     const int R = r0 + lane;
     const double QP = __ldg(a.bra.Q + P);
     const bool active = R < r1 && QP * __ldg(a.ket.Q + min(R, r1 - 1)) >= a.thresh;

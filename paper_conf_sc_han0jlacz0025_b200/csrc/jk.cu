@@ -37,6 +37,14 @@ mako_status launch_batch_class(int X, int Y, const BatchArgs& a, void* stream) {
   return fail(MAKO_ERR_UNSUPPORTED, "unknown class");
 }
 
+static int class_task_kets(int X, int Y) {
+#define MAKO_KT_CASE(x, y) \
+  if (X == x && Y == y) return task_kets_xy<x, y>();
+  MAKO_CLASS_LIST(MAKO_KT_CASE)
+#undef MAKO_KT_CASE
+  return 16;
+}
+
 static mako_status cuda_check(cudaError_t e, const char* what) {
   if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
   return MAKO_OK;
@@ -50,14 +58,14 @@ static mako_status upload(DevBuf& d, const std::vector<T>& h) {
   return MAKO_OK;
 }
 
-// number of kets R of bucket Y (Q-sorted desc) with QP * Q[R] >= thresh
-static int prefix_count(const std::vector<double>& QY, double QP, double thresh) {
-  int lo = 0, hi = (int)QY.size();
+// number of kets R in [lo, hi) of bucket Y (Q-sorted desc within the segment) with QP * Q[R] >= thresh
+static int prefix_count(const std::vector<double>& QY, int lo0, int hi0, double QP, double thresh) {
+  int lo = lo0, hi = hi0;
   while (lo < hi) {
     int mid = (lo + hi) / 2;
     if (QP * QY[mid] >= thresh) lo = mid + 1; else hi = mid;
   }
-  return lo;
+  return lo - lo0;
 }
 
 static mako_status ensure_plan(mako_pairs P, double thresh) {
@@ -71,22 +79,29 @@ static mako_status ensure_plan(mako_pairs P, double thresh) {
       ClassPlan& c = pl.cls[class_index(X, Y)];
       c.X = X;
       c.Y = Y;
-      c.KT = class_kt(X, Y);
+      c.KT = class_task_kets(X, Y);
       const PairBucket& bx = P->set.b[X];
       const PairBucket& by = P->set.b[Y];
-      const int nbra = bx.n();
-      c.nket.assign(nbra, 0);
-      c.task_off.assign(nbra + 1, 0);
-      for (int p = 0; p < nbra; ++p) {
-        int nk = by.n() ? prefix_count(by.Q, bx.Q[p], thresh) : 0;
-        if (X == Y) nk = std::min(nk, p + 1);
-        c.nket[p] = nk;
-        c.nquartet += nk;
-        c.task_off[p + 1] = c.task_off[p] + (nk + c.KT - 1) / c.KT;
-      }
-      c.ntask = c.task_off[nbra];
+      const int nbra = bx.n(), G = NKGROUP;
+      c.kbeg.assign((size_t)nbra * G, 0);
+      c.kend.assign((size_t)nbra * G, 0);
+      c.task_off.assign((size_t)nbra * G + 1, 0);
+      for (int p = 0; p < nbra; ++p)
+        for (int g = 0; g < G; ++g) {
+          const size_t u = (size_t)p * G + g;
+          const int s0 = by.seg.empty() ? 0 : by.seg[g], s1 = by.seg.empty() ? (g == 0 ? by.n() : 0) : by.seg[g + 1];
+          int nk = s1 > s0 ? prefix_count(by.Q, s0, s1, bx.Q[p], thresh) : 0;
+          if (X == Y) nk = std::min(nk, std::max(0, p - s0 + 1));  // canonical: ket position <= bra position
+          c.kbeg[u] = s0;
+          c.kend[u] = s0 + nk;
+          c.nquartet += nk;
+          c.task_off[u + 1] = c.task_off[u] + (nk + c.KT - 1) / c.KT;
+        }
+      c.ntask = c.task_off[(size_t)nbra * G];
       mako_status st;
-      if (c.ntask > 0 && ((st = upload(c.d_nket, c.nket)) || (st = upload(c.d_task_off, c.task_off)))) return st;
+      if (c.ntask > 0 && ((st = upload(c.d_kbeg, c.kbeg)) || (st = upload(c.d_kend, c.kend)) ||
+                          (st = upload(c.d_task_off, c.task_off))))
+        return st;
     }
   pl.thresh = thresh;
   return MAKO_OK;
@@ -181,13 +196,15 @@ static mako_status class_flops(mako_pairs p, double thresh, int shard, int nshar
     const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
     const double hab = nH(la + lb), hcd = nH(lc + ld);
     const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
-    // ket prefix of bra P restricted to this shard's tasks; by.poff is the prefix sum of K_CD
-    for (int P = 0; P < (int)c.nket.size(); ++P) {
-      const long long a0 = c.task_off[P], a1 = c.task_off[P + 1];
+    // surviving kets of each (bra, K-group) entry restricted to this shard's tasks
+    const int G = NKGROUP;
+    for (size_t u = 0; u < c.kbeg.size(); ++u) {
+      const long long a0 = c.task_off[u], a1 = c.task_off[u + 1];
       if (a1 <= t0 || a0 >= t1) continue;
-      const long long KAB = bx.poff[P + 1] - bx.poff[P];
-      const int r0 = (int)(std::max(a0, t0) - a0) * KT;
-      const int r1 = std::min((int)(std::min(a1, t1) - a0) * KT, c.nket[P]);
+      const int Pb = (int)(u / G);
+      const long long KAB = bx.poff[Pb + 1] - bx.poff[Pb];
+      const int r0 = c.kbeg[u] + (int)(std::max(a0, t0) - a0) * KT;
+      const int r1 = std::min(c.kbeg[u] + (int)(std::min(a1, t1) - a0) * KT, c.kend[u]);
       if (r1 <= r0) continue;
       const long long sumK = by.poff[r1] - by.poff[r0];
       fl[ci] += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)sumK * 2.0 * nab * hcd * ncd;
@@ -317,8 +334,10 @@ extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thres
       a.ket = p->set.b[c.Y].view();
       a.same_bucket = c.X == c.Y;
       a.task_off = c.d_task_off.as<long long>();
-      a.nket = c.d_nket.as<int>();
-      a.nbra = (int)c.nket.size();
+      a.kbeg = c.d_kbeg.as<int>();
+      a.kend = c.d_kend.as<int>();
+      a.nbra = (int)c.kbeg.size();
+      a.ngroup = NKGROUP;
       a.KT = c.KT;
       a.counter = p->d_counters.as<unsigned long long>() + class_index(c.X, c.Y);
       a.D = D;

@@ -62,6 +62,16 @@ MK_HD constexpr int tpq_regs(int X, int Y) {
 MK_HD constexpr bool use_tpq(int X, int Y) { return Y <= 1 && tpq_regs(X, Y) <= 100; }
 MK_HD constexpr int class_kt(int X, int Y) { return use_tpq(X, Y) ? 32 : 16; }
 
+// Pair buckets are ordered by (primitive-pair count group, Q descending): inside a group the
+// Schwarz-surviving kets of a bra are still a prefix, and the kets of one warp task share a similar
+// K_CD (uniform per-lane primitive loops).  Groups: K = 1, 2, 3, 4, 5-6, 7-9, 10-12, 13-16, 17-24,
+// 25-36, 37+.
+constexpr int NKGROUP = 11;
+MK_HD constexpr int kgroup(int K) {
+  return K <= 4 ? (K < 1 ? 0 : K - 1)
+                : (K <= 6 ? 4 : (K <= 9 ? 5 : (K <= 12 ? 6 : (K <= 16 ? 7 : (K <= 24 ? 8 : (K <= 36 ? 9 : 10))))));
+}
+
 // primitive-pair screening (reading R7)
 constexpr double PRIM_PAIR_EPS = 1e-18;
 
@@ -85,9 +95,11 @@ struct JKArgs {
   PairView bra, ket;
   int same_bucket;
   long long task_begin, task_end;   // shard range of this class's task index space
-  const long long* task_off;        // [nbra+1] task prefix per bra pair
-  const int* nket;                  // [nbra] kets per bra (prefix of the Q-sorted ket bucket)
-  int nbra;
+  const long long* task_off;        // [nbra+1] task prefix per flat (bra pair, ket K-group) entry
+  const int* kbeg;                  // [nbra] first ket of the entry (start of its K-group segment)
+  const int* kend;                  // [nbra] one past the last surviving ket (Q-sorted prefix of the segment)
+  int nbra;                         // flat entries = bra pairs x ngroup
+  int ngroup;                       // ket primitive-count groups per bucket
   int KT;                           // kets per task
   unsigned long long* counter;      // dynamic task counter (zeroed before launch)
   const double* D;

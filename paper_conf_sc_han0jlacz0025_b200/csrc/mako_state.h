@@ -43,6 +43,7 @@ struct PairBucket {
   std::vector<int> shA, shB;       // host copies
   std::vector<double> Q;           // host copy (sorted descending in a screened set)
   std::vector<int> poff;           // [n+1]
+  std::vector<int> seg;            // [NKGROUP+1] K-group segment starts (screened sets only)
   DevBuf d_shA, d_shB, d_Q, d_poff, d_pdat, d_Ebra, d_Eket;
   int n() const { return (int)shA.size(); }
   PairView view() const;
@@ -58,9 +59,9 @@ struct ClassPlan {
   int KT = 16;                     // kets per task
   long long ntask = 0;             // tasks of the whole class (all shards)
   long long nquartet = 0;
-  std::vector<int> nket;           // [nbra]
-  std::vector<long long> task_off; // [nbra+1]
-  DevBuf d_nket, d_task_off;
+  std::vector<int> kbeg, kend;     // [nbra * NKGROUP]
+  std::vector<long long> task_off; // [nbra * NKGROUP + 1]
+  DevBuf d_kbeg, d_kend, d_task_off;
 };
 
 struct Plan {

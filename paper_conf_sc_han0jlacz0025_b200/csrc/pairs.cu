@@ -258,17 +258,25 @@ extern "C" mako_status mako_shellpairs_screen(mako_basis basis, double thresh, v
     P->tau = thresh;
     std::vector<int> A2[NBUCKET], B2[NBUCKET];
     std::vector<double> Q2[NBUCKET];
+    std::vector<int> seg[NBUCKET];
     for (int b = 0; b < NBUCKET; ++b) {
       const PairBucket& cb = cand.b[b];
       std::vector<int> keep;
       for (int k = 0; k < cb.n(); ++k)
         if (cb.poff[k + 1] > cb.poff[k] && cb.Q[k] > 0 && cb.Q[k] * qmax >= thresh) keep.push_back(k);
-      std::stable_sort(keep.begin(), keep.end(), [&](int x, int y) { return cb.Q[x] > cb.Q[y]; });
+      auto grp = [&](int k) { return kgroup(cb.poff[k + 1] - cb.poff[k]); };
+      std::stable_sort(keep.begin(), keep.end(), [&](int x, int y) {
+        const int gx = grp(x), gy = grp(y);
+        return gx != gy ? gx < gy : cb.Q[x] > cb.Q[y];
+      });
+      seg[b].assign(NKGROUP + 1, 0);
       for (int k : keep) {
         A2[b].push_back(cb.shA[k]);
         B2[b].push_back(cb.shB[k]);
         Q2[b].push_back(cb.Q[k]);
+        seg[b][grp(k) + 1]++;
       }
+      for (int g = 0; g < NKGROUP; ++g) seg[b][g + 1] += seg[b][g];
     }
     for (int b = 0; b < NBUCKET; ++b) {  // free candidate device memory before the rebuild
       cand.b[b].d_Ebra.release();
@@ -278,6 +286,7 @@ extern "C" mako_status mako_shellpairs_screen(mako_basis basis, double thresh, v
     cudaStream_t s = (cudaStream_t)cuda_stream;
     for (int b = 0; b < NBUCKET; ++b) {
       P->set.b[b].Q = Q2[b];
+      P->set.b[b].seg = seg[b];
       if ((st = upload_async(P->set.b[b].d_Q, Q2[b], s))) return st;
     }
     if ((st = P->d_counters.alloc(sizeof(unsigned long long) * 64))) return st;
