@@ -182,11 +182,14 @@ void boys_table(std::vector<double>& tab) {
         }
       }
     }
-    for (int m = 0; m < BOYS_NM; ++m) tab[(size_t)k * BOYS_STRIDE + m] = (double)acc[m];
-    tab[(size_t)k * BOYS_STRIDE + BOYS_ECOL] = (double)expl(-T);
+    for (int L = 0; L < BOYS_LTAB; ++L) {
+      double* row = tab.data() + ((size_t)L * BOYS_NGRID + k) * BOYS_ROW;
+      for (int j = 0; j < BOYS_TAYLOR; ++j) row[j] = (double)acc[L + j];
+      row[BOYS_ROW - 1] = (double)expl(-T);
+    }
   }
   for (int k = 0; k < BOYS_NEXP; ++k)
-    tab[(size_t)BOYS_NGRID * BOYS_STRIDE + k] = (double)expl(-(40.0L + (long double)k * (long double)BOYS_H));
+    tab[BOYS_EXP_OFF + k] = (double)expl(-(40.0L + (long double)k * (long double)BOYS_H));
 }
 
 }  // namespace mako

@@ -113,15 +113,16 @@ __device__ __forceinline__ void boys_eval(double T, const double* __restrict__ t
   if (T < BOYS_TMAX) {
     const int k = __double2int_rn(T * (1.0 / BOYS_H));
     const double x = fma((double)k, BOYS_H, -T);
-    const double* r = tab + k * BOYS_STRIDE + L;
+    const double2* r = reinterpret_cast<const double2*>(tab + ((size_t)L * BOYS_NGRID + k) * BOYS_ROW);
+    const double2 r01 = __ldg(r), r23 = __ldg(r + 1), r45 = __ldg(r + 2), r6e = __ldg(r + 3);
     const double x2 = x * 0.5, x3 = x * (1.0 / 3.0), x4 = x * 0.25, x5 = x * 0.2, x6 = x * (1.0 / 6.0);
-    double f = __ldg(r + 6);
-    f = fma(f, x6, __ldg(r + 5));
-    f = fma(f, x5, __ldg(r + 4));
-    f = fma(f, x4, __ldg(r + 3));
-    f = fma(f, x3, __ldg(r + 2));
-    f = fma(f, x2, __ldg(r + 1));
-    f = fma(f, x, __ldg(r));
+    double f = r6e.x;
+    f = fma(f, x6, r45.y);
+    f = fma(f, x5, r45.x);
+    f = fma(f, x4, r23.y);
+    f = fma(f, x3, r23.x);
+    f = fma(f, x2, r01.y);
+    f = fma(f, x, r01.x);
     F[L] = f;
     if constexpr (L > 0) {
       double e = fma(x6, 1.0, 1.0);
@@ -130,7 +131,7 @@ __device__ __forceinline__ void boys_eval(double T, const double* __restrict__ t
       e = fma(e, x3, 1.0);
       e = fma(e, x2, 1.0);
       e = fma(e, x, 1.0);
-      e *= __ldg(tab + k * BOYS_STRIDE + BOYS_ECOL);
+      e *= r6e.y;
       const double t2 = 2.0 * T;
 #pragma unroll
       for (int m = L - 1; m >= 0; --m) F[m] = fma(t2, F[m + 1], e) * (1.0 / (2 * m + 1));
@@ -149,7 +150,7 @@ __device__ __forceinline__ void boys_eval(double T, const double* __restrict__ t
         s = fma(s, x * (1.0 / 3.0), 1.0);
         s = fma(s, x * 0.5, 1.0);
         s = fma(s, x, 1.0);
-        e = s * __ldg(tab + (size_t)BOYS_NGRID * BOYS_STRIDE + k);
+        e = s * __ldg(tab + BOYS_EXP_OFF + k);
       }
       const double h = 0.5 * rs * rs;
 #pragma unroll
@@ -208,6 +209,14 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
   }
 }
 
+// primitive-pair record {p, Px, Py, Pz} (32 B aligned): two 128-bit loads
+__device__ __forceinline__ void load_pdat(const double* __restrict__ pdat, int i, double& p, double& x, double& y,
+                                          double& z) {
+  const double2* v = reinterpret_cast<const double2*>(pdat + 4 * (size_t)i);
+  const double2 a = __ldg(v), b = __ldg(v + 1);
+  p = a.x; x = a.y; y = b.x; z = b.y;
+}
+
 __device__ __forceinline__ void dmma884(double& c0, double& c1, double a, double b) {
   asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
                : "+d"(c0), "+d"(c1)
@@ -230,16 +239,16 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
 #pragma unroll
       for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
     for (int kl = k0; kl < k1; ++kl) {
-      const double q = __ldg(ket.pdat + 4 * kl), Qx = __ldg(ket.pdat + 4 * kl + 1), Qy = __ldg(ket.pdat + 4 * kl + 2),
-                   Qz = __ldg(ket.pdat + 4 * kl + 3);
+      double q, Qx, Qy, Qz;
+      load_pdat(ket.pdat, kl, q, Qx, Qy, Qz);
       double t1[C::MC][C::NT1][2];
 #pragma unroll
       for (int mc = 0; mc < C::MC; ++mc)
 #pragma unroll
         for (int nt = 0; nt < C::NT1; ++nt) t1[mc][nt][0] = t1[mc][nt][1] = 0.0;
       for (int ij = b0; ij < b1; ++ij) {
-        const double p = __ldg(bra.pdat + 4 * ij), Px = __ldg(bra.pdat + 4 * ij + 1),
-                     Py = __ldg(bra.pdat + 4 * ij + 2), Pz = __ldg(bra.pdat + 4 * ij + 3);
+        double p, Px, Py, Pz;
+        load_pdat(bra.pdat, ij, p, Px, Py, Pz);
         compute_R<C>(p, Px, Py, Pz, q, Qx, Qy, Qz, Rbuf, rtab, btab, lane);
         const double* __restrict__ E = bra.Ebra + (size_t)ij * (C::NAB * C::NHAB);
 #pragma unroll

@@ -18,6 +18,8 @@ template <int X, int Y>
 int jk_blocks_per_sm();
 template <int X, int Y>
 int task_kets_xy();
+template <int X, int Y>
+bool swap_xy();
 
 }  // namespace mako
 
@@ -147,7 +149,11 @@ int jk_blocks_per_sm() {
   static int cached = -1;
   if (cached < 0) {
     int nb = 0;
-    if constexpr (use_kf<X, Y>()) {
+    if constexpr (use_kf_swap<X, Y>()) {
+      constexpr size_t ks = KfCfg<Y, X>::SMEM;
+      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel<Y, X>, ks)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel<Y, X>, CTA_THREADS, ks);
+    } else if constexpr (use_kf<X, Y>()) {
       constexpr size_t ks = KfCfg<X, Y>::SMEM;
       if (set_smem_attr<X, Y>((const void*)kf_jk_kernel<X, Y>, ks)) return 1;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel<X, Y>, CTA_THREADS, ks);
@@ -177,9 +183,12 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   const int bps = jk_blocks_per_sm<X, Y>();
   long long want = (ntask + CTA_WARPS - 1) / CTA_WARPS;
-  long long cap = (long long)nsm * bps;
+  long long cap = (long long)nsm * bps / (a.grid_div > 1 ? a.grid_div : 1);
+  if (cap < nsm) cap = nsm;
   const int grid = (int)(want < cap ? want : cap);
-  if constexpr (use_kf<X, Y>())
+  if constexpr (use_kf_swap<X, Y>())
+    kf_jk_kernel<Y, X><<<grid, CTA_THREADS, KfCfg<Y, X>::SMEM, (cudaStream_t)stream>>>(a);
+  else if constexpr (use_kf<X, Y>())
     kf_jk_kernel<X, Y><<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
   else if constexpr (use_tpq(X, Y))
     tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, (cudaStream_t)stream>>>(a);
@@ -213,9 +222,14 @@ mako_status launch_batch_xy(const BatchArgs& a, void* stream) {
 namespace mako {
 template <int X, int Y>
 int task_kets_xy() {
-  if constexpr (use_kf<X, Y>()) return KfCfg<X, Y>::NK;
+  if constexpr (use_kf_swap<X, Y>()) return KfCfg<Y, X>::NK;
+  else if constexpr (use_kf<X, Y>()) return KfCfg<X, Y>::NK;
   else if constexpr (use_tpq(X, Y)) return 32;
   else return 16;
+}
+template <int X, int Y>
+bool swap_xy() {
+  return use_kf_swap<X, Y>();
 }
 }  // namespace mako
 
@@ -223,5 +237,6 @@ int task_kets_xy() {
   template mako_status mako::launch_jk_xy<X, Y>(const mako::JKArgs&, void*, int*);               \
   template mako_status mako::launch_batch_xy<X, Y>(const mako::BatchArgs&, void*);               \
   template int mako::jk_blocks_per_sm<X, Y>();                                                   \
-  template int mako::task_kets_xy<X, Y>();
+  template int mako::task_kets_xy<X, Y>();                                                       \
+  template bool mako::swap_xy<X, Y>();
 #endif

@@ -37,7 +37,7 @@ struct KfCfg {
   static constexpr int ROWS = (C::MT * 8 > C::KS1 * 4) ? C::MT * 8 : C::KS1 * 4;
   static constexpr int WARP_DBL = ROWS * WS;
   static constexpr size_t SMEM = sizeof(double) * 4 * WARP_DBL;
-  static constexpr bool OK = NK > 0 && Y <= 3 && C::L <= 6;
+  static constexpr bool OK = NK > 0 && C::NHCD * C::NCD <= 140 && C::L <= 6;
 };
 
 template <int X, int Y>
@@ -48,6 +48,17 @@ constexpr bool use_kf() {
   constexpr bool pick = c == 303 || c == 401 || c == 403 || c == 501 || c == 603 || c == 701 || c == 800 ||
                         c == 801 || c == 900 || c == 700 || c == 500;
   return KfCfg<X, Y>::OK && pick;
+}
+
+// Transposed execution of class (X|Y), X > Y: the task pair comes from bucket Y and the lanes take
+// pairs of bucket X, i.e. kf_jk_kernel<Y, X> computes (cd|ab) = (ab|cd) (8-fold symmetry) with the
+// lighter side contracted per lane.  Used when the canonical ket has more functions than the bra.
+template <int X, int Y>
+constexpr bool use_kf_swap() {
+  constexpr int c = X * 100 + Y;
+  constexpr bool pick = c == 302;
+  if constexpr (X != Y) return KfCfg<Y, X>::OK && pick;
+  return false;
 }
 
 template <int X, int Y>
@@ -91,16 +102,16 @@ __global__ void __launch_bounds__(128) kf_jk_kernel(JKArgs a) {
       for (int n = 0; n < NTV; ++n) vf[m][n][0] = vf[m][n][1] = 0.0;
     for (int ij = b0; ij < b1; ++ij) {
       // ---- DFMA stage: this lane's p-slice of W^{ij} for its ket ----
-      const double p = __ldg(a.bra.pdat + 4 * ij), Px = __ldg(a.bra.pdat + 4 * ij + 1),
-                   Py = __ldg(a.bra.pdat + 4 * ij + 2), Pz = __ldg(a.bra.pdat + 4 * ij + 3);
+      double p, Px, Py, Pz;
+        load_pdat(a.bra.pdat, ij, p, Px, Py, Pz);
       double W[PP][NCD];
 #pragma unroll
       for (int i = 0; i < PP; ++i)
 #pragma unroll
         for (int j = 0; j < NCD; ++j) W[i][j] = 0.0;
       for (int kl = k0; kl < k1; ++kl) {
-        const double q = __ldg(a.ket.pdat + 4 * kl), Qx = __ldg(a.ket.pdat + 4 * kl + 1),
-                     Qy = __ldg(a.ket.pdat + 4 * kl + 2), Qz = __ldg(a.ket.pdat + 4 * kl + 3);
+        double q, Qx, Qy, Qz;
+        load_pdat(a.ket.pdat, kl, q, Qx, Qy, Qz);
         double Rr[nH(L)];
         r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
         const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);

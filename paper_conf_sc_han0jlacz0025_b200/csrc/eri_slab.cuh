@@ -151,10 +151,10 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
 #pragma unroll
           for (int z = 0; z < NS; ++z)
             if (z == s) klc = s_kl[z];
-          const double p = __ldg(a.bra.pdat + 4 * ij), Px = __ldg(a.bra.pdat + 4 * ij + 1),
-                       Py = __ldg(a.bra.pdat + 4 * ij + 2), Pz = __ldg(a.bra.pdat + 4 * ij + 3);
-          const double q = __ldg(a.ket.pdat + 4 * klc), Qx = __ldg(a.ket.pdat + 4 * klc + 1),
-                       Qy = __ldg(a.ket.pdat + 4 * klc + 2), Qz = __ldg(a.ket.pdat + 4 * klc + 3);
+          double p, Px, Py, Pz;
+        load_pdat(a.bra.pdat, ij, p, Px, Py, Pz);
+          double q, Qx, Qy, Qz;
+        load_pdat(a.ket.pdat, klc, q, Qx, Qy, Qz);
           double Rr[nH(L)];
           r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
           double* row = Rs + (size_t)c * RS;

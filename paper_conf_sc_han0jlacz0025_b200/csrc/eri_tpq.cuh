@@ -44,6 +44,25 @@ __device__ __forceinline__ void static_for(F&& f) {
   }
 }
 
+// NH x NC doubles (contiguous, 16 B aligned when NH*NC is even) into a register matrix
+template <int NH, int NC>
+__device__ __forceinline__ void load_mat(const double* __restrict__ src, double (&M)[NH][NC]) {
+  if constexpr ((NH * NC) % 2 == 0) {
+    const double2* v = reinterpret_cast<const double2*>(src);
+    static_for<0, NH * NC / 2>([&](auto ic) {
+      constexpr int i = decltype(ic)::value;
+      const double2 w = __ldg(v + i);
+      M[(2 * i) / NC][(2 * i) % NC] = w.x;
+      M[(2 * i + 1) / NC][(2 * i + 1) % NC] = w.y;
+    });
+  } else {
+#pragma unroll
+    for (int h = 0; h < NH; ++h)
+#pragma unroll
+      for (int j = 0; j < NC; ++j) M[h][j] = __ldg(src + h * NC + j);
+  }
+}
+
 // one level of the in-place R recursion: entries E, E-1, ..., 1 (descending = degree-descending,
 // so every source of level n+1 is still unmodified when read)
 template <int E>
@@ -146,22 +165,19 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
       if constexpr (WACC) {
         // bra primitive outer: W[p][cd] = sum_kl sum_q R_{p+q} E~_cd[q][cd], then V += E~_ab W
         for (int ij = b0; ij < b1; ++ij) {
-          const double p = __ldg(a.bra.pdat + 4 * ij), Px = __ldg(a.bra.pdat + 4 * ij + 1),
-                       Py = __ldg(a.bra.pdat + 4 * ij + 2), Pz = __ldg(a.bra.pdat + 4 * ij + 3);
+          double p, Px, Py, Pz;
+        load_pdat(a.bra.pdat, ij, p, Px, Py, Pz);
           double W[NHAB][NCD];
 #pragma unroll
           for (int h = 0; h < NHAB; ++h)
 #pragma unroll
             for (int j = 0; j < NCD; ++j) W[h][j] = 0.0;
           for (int kl = k0; kl < k1; ++kl) {
-            const double q = __ldg(a.ket.pdat + 4 * kl), Qx = __ldg(a.ket.pdat + 4 * kl + 1),
-                         Qy = __ldg(a.ket.pdat + 4 * kl + 2), Qz = __ldg(a.ket.pdat + 4 * kl + 3);
+            double q, Qx, Qy, Qz;
+        load_pdat(a.ket.pdat, kl, q, Qx, Qy, Qz);
             double Ek[NHCD][NCD];
             const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
-#pragma unroll
-            for (int h = 0; h < NHCD; ++h)
-#pragma unroll
-              for (int j = 0; j < NCD; ++j) Ek[h][j] = __ldg(ek + h * NCD + j);
+            load_mat<NHCD, NCD>(ek, Ek);
             double Rr[nH(L)];
             r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
             static_for<0, NHAB>([&](auto pc) {
@@ -186,18 +202,15 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
         }
       } else {
       for (int kl = k0; kl < k1; ++kl) {
-        const double q = __ldg(a.ket.pdat + 4 * kl), Qx = __ldg(a.ket.pdat + 4 * kl + 1),
-                     Qy = __ldg(a.ket.pdat + 4 * kl + 2), Qz = __ldg(a.ket.pdat + 4 * kl + 3);
+        double q, Qx, Qy, Qz;
+        load_pdat(a.ket.pdat, kl, q, Qx, Qy, Qz);
         // signed ket E~^T [q][cd]
         double Ek[NHCD][NCD];
         const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
-#pragma unroll
-        for (int h = 0; h < NHCD; ++h)
-#pragma unroll
-          for (int j = 0; j < NCD; ++j) Ek[h][j] = __ldg(ek + h * NCD + j);
+        load_mat<NHCD, NCD>(ek, Ek);
         for (int ij = b0; ij < b1; ++ij) {
-          const double p = __ldg(a.bra.pdat + 4 * ij), Px = __ldg(a.bra.pdat + 4 * ij + 1),
-                       Py = __ldg(a.bra.pdat + 4 * ij + 2), Pz = __ldg(a.bra.pdat + 4 * ij + 3);
+          double p, Px, Py, Pz;
+        load_pdat(a.bra.pdat, ij, p, Px, Py, Pz);
           double Rr[nH(L)];
           r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
           const double* __restrict__ eb = a.bra.Ebra + (size_t)ij * (NAB * NHAB);

@@ -42,12 +42,15 @@ constexpr int BOYS_NGRID = 1281;      // T_k up to 40
 constexpr int BOYS_MMAX = 24;         // supports L + 6 <= 24
 constexpr int BOYS_NM = BOYS_MMAX + 1;
 constexpr int BOYS_TAYLOR = 7;        // Taylor terms (|dT| <= 1/64 -> truncation < 5e-17 relative)
-constexpr int BOYS_STRIDE = 32;       // row stride (doubles); column BOYS_ECOL holds exp(-T_k)
-constexpr int BOYS_ECOL = 31;
+// per-L packed rows: block L (0 <= L < BOYS_LTAB), row k = {F_L..F_{L+6}(T_k), exp(-T_k)}: 64 B,
+// read with four 128-bit loads (one cache line per lane and lookup)
+constexpr int BOYS_LTAB = BOYS_MMAX - BOYS_TAYLOR + 2;  // L = 0..18
+constexpr int BOYS_ROW = 8;
 constexpr double BOYS_TEXP = 80.0;    // for 40 <= T < 80 exp(-T) comes from a second grid; beyond, it is
                                       // below 1e-18 of every F_m (m <= 12) and is dropped (reading R1)
 constexpr int BOYS_NEXP = 1281;       // exp(-(40 + k/32)), k = 0..1280
-constexpr size_t BOYS_TABLE_DOUBLES = (size_t)BOYS_NGRID * BOYS_STRIDE + BOYS_NEXP;
+constexpr size_t BOYS_EXP_OFF = (size_t)BOYS_LTAB * BOYS_NGRID * BOYS_ROW;
+constexpr size_t BOYS_TABLE_DOUBLES = BOYS_EXP_OFF + BOYS_NEXP;
 
 // Kernel family per class (X >= Y buckets).  Low-l classes use the lane-per-ket register kernel
 // ("TPQ": Boys, R, contraction and digestion in registers of one lane), the rest the warp-per-quartet
@@ -109,6 +112,7 @@ struct JKArgs {
   const int* ao;                    // [nshell] AO offsets
   double thresh;
   const double* boys;               // Boys table
+  int grid_div;                     // host side: grid = resident capacity / grid_div (concurrent classes)
 };
 
 // arguments of a store/diag class launch (eri_batch, Schwarz)

@@ -57,6 +57,8 @@ struct PairSet {
 struct ClassPlan {
   int X = 0, Y = 0;                // bra / ket buckets (X >= Y)
   int KT = 16;                     // kets per task
+  bool swap = false;               // transposed execution: task pairs from bucket Y, lanes from X
+  int TB = 0, LB = 0;              // task bucket, lane bucket
   long long ntask = 0;             // tasks of the whole class (all shards)
   long long nquartet = 0;
   std::vector<int> kbeg, kend;     // [nbra * NKGROUP]
@@ -93,6 +95,10 @@ struct mako_pairs_s {
   mako::DevBuf d_counters;      // [55] task counters
   // profiling (mako_profile_enable / read)
   bool prof = false;
+  // concurrent class launches: internal streams forked from / joined to the caller's stream
+  std::vector<void*> streams;       // cudaStream_t
+  void* ev_fork = nullptr;          // cudaEvent_t
+  std::vector<void*> ev_join;       // cudaEvent_t per internal stream
   std::vector<std::pair<int, std::pair<void*, void*>>> prof_events;  // (class, (start, stop)) cudaEvent_t
   ~mako_pairs_s();
 };
