@@ -47,7 +47,8 @@ struct Cls {
   static constexpr int W_R = 2 * NH;    // ping-pong R levels
   static constexpr int W_V = NAB * NCD; // (ab|cd) block
   static constexpr int W_J = NAB;       // J_ab partial sums over the kets of a task
-  static constexpr int WARP_DBL = W_R + W_V + W_J;
+  static constexpr int W_D = NA * NB + NC * ND + NA * NC + NA * ND + NB * NC + NB * ND;  // staged D blocks
+  static constexpr int WARP_DBL = W_R + W_V + W_J + W_D;
   // CTA tables
   static constexpr int HTAB_BYTES = ((NHAB * NHCD * 2 + 15) / 16) * 16;
   static constexpr int RTAB_BYTES = ((NH * 4 + 15) / 16) * 16;
@@ -305,62 +306,107 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
 // With v' = deg * (ab|cd), deg = 1/2 per coincidence (a=b, c=d, ab=cd), the 8 permutations of a
 // canonical quartet reduce for symmetric D to the 6 forward updates below; the transposed halves
 // are restored by J = Jacc + Jacc^T, K = Kacc + Kacc^T at the end of the build.
+// The six D sub-blocks are first staged in warp SMEM (Ds, DIGEST_DS doubles) with coalesced row
+// loads, so the reduction loops below run on SMEM with two independent accumulators.
+template <class C>
+struct DigestLayout {
+  static constexpr int AB = 0, CD = AB + C::NA * C::NB, AC = CD + C::NC * C::ND, AD = AC + C::NA * C::NC,
+                       BC = AD + C::NA * C::ND, BD = BC + C::NB * C::NC, TOT = BD + C::NB * C::ND;
+};
+constexpr int DIGEST_DS = 6 * 49;
+
 template <class C>
 __device__ void digest(const double* __restrict__ V, double deg, int oa, int ob, int oc, int od,
                        const double* __restrict__ D, int nbf, double* __restrict__ J, double* __restrict__ K,
-                       double* __restrict__ jab, int lane) {
+                       double* __restrict__ jab, double* __restrict__ Ds, int lane) {
+  using DL = DigestLayout<C>;
+  constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND, NCD = C::NCD;
+  // stage D_ab, D_cd, D_ac, D_ad, D_bc, D_bd
+  for (int x = lane; x < DL::TOT; x += 32) {
+    int r, c;
+    if (x < DL::CD) { r = oa + (x - DL::AB) / NB; c = ob + (x - DL::AB) % NB; }
+    else if (x < DL::AC) { r = oc + (x - DL::CD) / ND; c = od + (x - DL::CD) % ND; }
+    else if (x < DL::AD) { r = oa + (x - DL::AC) / NC; c = oc + (x - DL::AC) % NC; }
+    else if (x < DL::BC) { r = oa + (x - DL::AD) / ND; c = od + (x - DL::AD) % ND; }
+    else if (x < DL::BD) { r = ob + (x - DL::BC) / NC; c = oc + (x - DL::BC) % NC; }
+    else { r = ob + (x - DL::BD) / ND; c = od + (x - DL::BD) % ND; }
+    Ds[x] = __ldg(D + (size_t)r * nbf + c);
+  }
+  __syncwarp();
+  const double* Dab = Ds + DL::AB;
+  const double* Dcd = Ds + DL::CD;
+  const double* Dac = Ds + DL::AC;
+  const double* Dad = Ds + DL::AD;
+  const double* Dbc = Ds + DL::BC;
+  const double* Dbd = Ds + DL::BD;
   // J_ab (accumulated in SMEM across the kets of the task)
   for (int ab = lane; ab < C::NAB; ab += 32) {
-    double s = 0.0;
-#pragma unroll 4
-    for (int cd = 0; cd < C::NCD; ++cd)
-      s = fma(V[ab * C::NCD + cd], __ldg(D + (size_t)(oc + cd / C::ND) * nbf + od + cd % C::ND), s);
-    jab[ab] = fma(2.0 * deg, s, jab[ab]);
+    double s0 = 0.0, s1 = 0.0;
+    int cd = 0;
+    for (; cd + 1 < NCD; cd += 2) {
+      s0 = fma(V[ab * NCD + cd], Dcd[cd], s0);
+      s1 = fma(V[ab * NCD + cd + 1], Dcd[cd + 1], s1);
+    }
+    if (cd < NCD) s0 = fma(V[ab * NCD + cd], Dcd[cd], s0);
+    jab[ab] = fma(2.0 * deg, s0 + s1, jab[ab]);
   }
   // J_cd
-  for (int cd = lane; cd < C::NCD; cd += 32) {
-    double s = 0.0;
-#pragma unroll 4
-    for (int ab = 0; ab < C::NAB; ++ab)
-      s = fma(V[ab * C::NCD + cd], __ldg(D + (size_t)(oa + ab / C::NB) * nbf + ob + ab % C::NB), s);
-    atomicAdd(J + (size_t)(oc + cd / C::ND) * nbf + od + cd % C::ND, 2.0 * deg * s);
+  for (int cd = lane; cd < NCD; cd += 32) {
+    double s0 = 0.0, s1 = 0.0;
+    int ab = 0;
+    for (; ab + 1 < C::NAB; ab += 2) {
+      s0 = fma(V[ab * NCD + cd], Dab[ab], s0);
+      s1 = fma(V[(ab + 1) * NCD + cd], Dab[ab + 1], s1);
+    }
+    if (ab < C::NAB) s0 = fma(V[ab * NCD + cd], Dab[ab], s0);
+    atomicAdd(J + (size_t)(oc + cd / ND) * nbf + od + cd % ND, 2.0 * deg * (s0 + s1));
   }
-  // K_ac += v D_bd
-  for (int x = lane; x < C::NA * C::NC; x += 32) {
-    const int i = x / C::NC, k = x % C::NC;
-    double s = 0.0;
-    for (int j = 0; j < C::NB; ++j)
-      for (int l = 0; l < C::ND; ++l)
-        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(ob + j) * nbf + od + l), s);
-    atomicAdd(K + (size_t)(oa + i) * nbf + oc + k, deg * s);
+  // K_ac += v D_bd | K_ad += v D_bc | K_bc += v D_ad | K_bd += v D_ac   (one flattened index space)
+  constexpr int N1 = NA * NC, N2 = N1 + NA * ND, N3 = N2 + NB * NC, N4 = N3 + NB * ND;
+  for (int x = lane; x < N4; x += 32) {
+    double s0 = 0.0, s1 = 0.0;
+    size_t dst;
+    double* Kp = K;
+    if (x < N1) {
+      const int i = x / NC, k = x % NC;
+      for (int j = 0; j < NB; ++j)
+#pragma unroll
+        for (int l = 0; l < ND; ++l) {
+          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dbd[j * ND + l];
+          if (l & 1) s1 += t; else s0 += t;
+        }
+      dst = (size_t)(oa + i) * nbf + oc + k;
+    } else if (x < N2) {
+      const int y = x - N1, i = y / ND, l = y % ND;
+      for (int j = 0; j < NB; ++j)
+#pragma unroll
+        for (int k = 0; k < NC; ++k) {
+          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dbc[j * NC + k];
+          if (k & 1) s1 += t; else s0 += t;
+        }
+      dst = (size_t)(oa + i) * nbf + od + l;
+    } else if (x < N3) {
+      const int y = x - N2, j = y / NC, k = y % NC;
+      for (int i = 0; i < NA; ++i)
+#pragma unroll
+        for (int l = 0; l < ND; ++l) {
+          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dad[i * ND + l];
+          if (l & 1) s1 += t; else s0 += t;
+        }
+      dst = (size_t)(ob + j) * nbf + oc + k;
+    } else {
+      const int y = x - N3, j = y / ND, l = y % ND;
+      for (int i = 0; i < NA; ++i)
+#pragma unroll
+        for (int k = 0; k < NC; ++k) {
+          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dac[i * NC + k];
+          if (k & 1) s1 += t; else s0 += t;
+        }
+      dst = (size_t)(ob + j) * nbf + od + l;
+    }
+    atomicAdd(Kp + dst, deg * (s0 + s1));
   }
-  // K_ad += v D_bc
-  for (int x = lane; x < C::NA * C::ND; x += 32) {
-    const int i = x / C::ND, l = x % C::ND;
-    double s = 0.0;
-    for (int j = 0; j < C::NB; ++j)
-      for (int k = 0; k < C::NC; ++k)
-        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(ob + j) * nbf + oc + k), s);
-    atomicAdd(K + (size_t)(oa + i) * nbf + od + l, deg * s);
-  }
-  // K_bc += v D_ad
-  for (int x = lane; x < C::NB * C::NC; x += 32) {
-    const int j = x / C::NC, k = x % C::NC;
-    double s = 0.0;
-    for (int i = 0; i < C::NA; ++i)
-      for (int l = 0; l < C::ND; ++l)
-        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(oa + i) * nbf + od + l), s);
-    atomicAdd(K + (size_t)(ob + j) * nbf + oc + k, deg * s);
-  }
-  // K_bd += v D_ac
-  for (int x = lane; x < C::NB * C::ND; x += 32) {
-    const int j = x / C::ND, l = x % C::ND;
-    double s = 0.0;
-    for (int i = 0; i < C::NA; ++i)
-      for (int k = 0; k < C::NC; ++k)
-        s = fma(V[(i * C::NB + j) * C::NCD + k * C::ND + l], __ldg(D + (size_t)(oa + i) * nbf + oc + k), s);
-    atomicAdd(K + (size_t)(ob + j) * nbf + od + l, deg * s);
-  }
+  __syncwarp();
 }
 
 }  // namespace mako

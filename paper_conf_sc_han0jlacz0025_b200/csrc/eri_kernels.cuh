@@ -76,7 +76,7 @@ __global__ void __launch_bounds__(CTA_THREADS) jk_kernel(JKArgs a) {
       if (sa == sb) deg *= 0.5;
       if (sc == sd) deg *= 0.5;
       if (a.same_bucket && P == R) deg *= 0.5;
-      digest<C>(V, deg, oa, ob, __ldg(a.ao + sc), __ldg(a.ao + sd), a.D, a.nbf, a.J, a.K, jab, lane);
+      digest<C>(V, deg, oa, ob, __ldg(a.ao + sc), __ldg(a.ao + sd), a.D, a.nbf, a.J, a.K, jab, jab + C::NAB, lane);
       __syncwarp();
     }
     for (int ab = lane; ab < C::NAB; ab += 32)

@@ -39,7 +39,7 @@ struct SlabCfg {
   // warp SMEM (doubles): R rows, V for NS kets, J_ab partial
   static constexpr int W_R = RCAP * RSTRIDE;
   static constexpr int W_V = NS * C::NAB * C::NCD;
-  static constexpr int WARP_DBL = W_R + W_V + C::NAB + 2;
+  static constexpr int WARP_DBL = W_R + W_V + C::NAB + 2 + C::W_D;
   // CTA table: B-fragment offsets [KS1][NT1B][32] (slot << 10 | hermite index, -1 = zero)
   static constexpr int HOFS_INTS = C::KS1 * NT1B * 32;
   static constexpr size_t SMEM = sizeof(int) * HOFS_INTS + sizeof(double) * 4 * WARP_DBL;
@@ -242,7 +242,7 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
         if (sc == sd) deg *= 0.5;
         if (a.same_bucket && P == R) deg *= 0.5;
         digest<C>(Vs + (size_t)v * NAB * NCD, deg, oa, ob, __ldg(a.ao + sc), __ldg(a.ao + sd), a.D, a.nbf, a.J, a.K,
-                  jab, lane);
+                  jab, jab + NAB + 2, lane);
         __syncwarp();
       }
     }
