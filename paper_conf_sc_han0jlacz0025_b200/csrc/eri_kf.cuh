@@ -38,6 +38,9 @@ struct KfCfg {
   static constexpr int WARP_DBL = ROWS * WS;
   static constexpr size_t SMEM = sizeof(double) * 4 * WARP_DBL;
   static constexpr bool OK = NK > 0 && C::NHCD * C::NCD <= 140 && C::L <= 6;
+  // 3 CTAs/SM (<= 168 registers, some spills) measured faster for these instantiations, else no cap
+  static constexpr int MINB = (X * 10 + Y == 41 || X * 10 + Y == 23 || X * 10 + Y == 71 || X * 10 + Y == 80 ||
+                               X * 10 + Y == 33 || X * 10 + Y == 90) ? 3 : 1;
 };
 
 template <int X, int Y>
@@ -62,7 +65,7 @@ constexpr bool use_kf_swap() {
 }
 
 template <int X, int Y>
-__global__ void __launch_bounds__(128) kf_jk_kernel(JKArgs a) {
+__global__ void __launch_bounds__(128, KfCfg<X, Y>::MINB) kf_jk_kernel(JKArgs a) {
   using C = ClsXY<X, Y>;
   using K = KfCfg<X, Y>;
   constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
