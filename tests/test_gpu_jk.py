@@ -115,3 +115,28 @@ def test_gly10_sampled_blocks():
         gk = K[off[x]:off[x + 1], off[y]:off[y + 1]]
         assert np.abs(gj - jb).max() <= 1e-8, (x, y, np.abs(gj - jb).max())
         assert np.abs(gk - kb).max() <= 1e-8, (x, y, np.abs(gk - kb).max())
+
+
+def test_valinomycin_full_size_sampled_blocks():
+    """The bench workload (valinomycin-sized def2-TZVP-shaped, tau = 1e-12, the same build call bench.py
+    times): exact J/K blocks of sampled shell pairs vs the oracle's definition-level blocks."""
+    tau = 1e-12
+    m, sh, B, P = _setup("valinomycin-def2tzvp", tau)
+    D = mi.synthetic_density(sh.nbf(), m.nelec // 2, seed=0)
+    J, K = _gpu_jk(P, D)
+    assert np.array_equal(J, J.T) and np.array_equal(K, K.T)
+    rng = np.random.default_rng(7)
+    # same-atom shell pairs (significant pairs, non-trivial J and K blocks), s-p and d-f
+    atoms = [int(a) for a in rng.choice(np.unique(sh.atom[sh.l == 3]), 2, replace=False)]
+    def on(a, l):
+        return [i for i in range(sh.nshell) if sh.atom[i] == a and sh.l[i] == l][0]
+    pairs = [(on(atoms[0], 0), on(atoms[0], 1)), (on(atoms[1], 2), on(atoms[1], 3))]
+    Q = oracle.schwarz(sh)
+    Jb, Kb = oracle.jk_blocks(sh, D, pairs, tau=tau, Q=Q)
+    off = B.ao_offsets
+    for (x, y), jb, kb in zip(pairs, Jb, Kb):
+        gj = J[off[x]:off[x + 1], off[y]:off[y + 1]]
+        gk = K[off[x]:off[x + 1], off[y]:off[y + 1]]
+        print("valinomycin block", x, y, np.abs(jb).max(), np.abs(kb).max(), np.abs(gj - jb).max(), np.abs(gk - kb).max())
+        assert np.abs(jb).max() > 1e-3 and np.abs(kb).max() > 1e-6
+        assert np.abs(gj - jb).max() <= 1e-8 and np.abs(gk - kb).max() <= 1e-8
