@@ -44,7 +44,10 @@ struct Cls {
   static constexpr int NCHUNK = (MT + MCMAX - 1) / MCMAX;
   static constexpr int MC = (MT + NCHUNK - 1) / NCHUNK;
   // per-warp shared memory (doubles)
-  static constexpr int W_R = 2 * NH;    // ping-pong R levels
+  // R rows kept per bra primitive (computed once per primitive quartet, reused by every row chunk)
+  // (d/f x d/f bra pairs are single-primitive in the def2/cc families: no rows to group)
+  static constexpr int KR = (LA >= 2 && LB >= 2) ? 1 : clampi(1200 / NH - 1, 1, 4);
+  static constexpr int W_R = (KR + 1) * NH;  // KR result rows + 1 ping-pong scratch row
   static constexpr int W_V = NAB * NCD; // (ab|cd) block
   static constexpr int W_J = NAB;       // J_ab partial sums over the kets of a task
   static constexpr int W_D = NA * NB + NC * ND + NA * NC + NA * ND + NB * NC + NB * ND;  // staged D blocks
@@ -166,8 +169,9 @@ __device__ __forceinline__ void boys_eval(double T, const double* __restrict__ t
 // Level n holds all entries with t+u+v <= L-n; lanes split each level; levels ping-pong.
 template <class C>
 __device__ __forceinline__ void compute_R(double p, double Px, double Py, double Pz, double q, double Qx, double Qy,
-                                          double Qz, double* __restrict__ buf, const uint32_t* __restrict__ rtab,
-                                          const double* __restrict__ btab, int lane) {
+                                          double Qz, double* __restrict__ dst, double* __restrict__ scratch,
+                                          const uint32_t* __restrict__ rtab, const double* __restrict__ btab,
+                                          int lane) {
   constexpr int L = C::L, NH = C::NH;
   const double pq = p + q, ri = rsqrt_fast(pq), rho = p * q * ri * ri;
   const double X = Px - Qx, Y = Py - Qy, Z = Pz - Qz;
@@ -182,15 +186,15 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
     s *= m2r;
   }
   if constexpr (L == 0) {
-    if (lane == 0) buf[0] = F[0];
+    if (lane == 0) dst[0] = F[0];
     __syncwarp();
   } else {
-    if (lane == 0) buf[(L & 1) * NH] = F[L];
+    if (lane == 0) ((L & 1) ? scratch : dst)[0] = F[L];
     __syncwarp();
 #pragma unroll
     for (int n = L - 1; n >= 0; --n) {
-      double* cur = buf + (n & 1) * NH;
-      const double* prv = buf + ((n + 1) & 1) * NH;
+      double* cur = (n & 1) ? scratch : dst;  // level 0 lands in dst
+      const double* prv = ((n + 1) & 1) ? scratch : dst;
       const int cnt = nH(L - n);
       for (int e = lane; e < cnt; e += 32) {
         double v;
@@ -226,78 +230,112 @@ __device__ __forceinline__ void dmma884(double& c0, double& c1, double a, double
 
 // (ab|cd) block for bra pair P of `bra` and ket pair R of `ket` into V[ab][cd] (warp SMEM).
 // m8n8k4 f64 fragments (lane = 4g + t): A[g][t]; B[k=t][n=g]; C[g][2t+i].
+// Per ket primitive: R is computed once for up to KR bra primitives into SMEM rows; every row chunk
+// (MC m-tiles, bounded by the accumulator register budget) then runs GEMM1 over those rows and the
+// register-chained GEMM2, and adds its rows of (ab|cd) into V.
 template <class C>
 __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, int R, double* __restrict__ Rbuf,
                               double* __restrict__ V, const uint16_t* __restrict__ htab,
                               const uint32_t* __restrict__ rtab, const double* __restrict__ btab, int lane) {
+  constexpr int KR = C::KR, NH = C::NH;
   const int g = lane >> 2, t = lane & 3;
   const int b0 = __ldg(bra.poff + P), b1 = __ldg(bra.poff + P + 1);
   const int k0 = __ldg(ket.poff + R), k1 = __ldg(ket.poff + R + 1);
-  for (int ch = 0; ch < C::NCHUNK; ++ch) {
-    double c2[C::MC][C::NT2][2];
-#pragma unroll
-    for (int mc = 0; mc < C::MC; ++mc)
-#pragma unroll
-      for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
-    for (int kl = k0; kl < k1; ++kl) {
-      double q, Qx, Qy, Qz;
-      load_pdat(ket.pdat, kl, q, Qx, Qy, Qz);
-      double t1[C::MC][C::NT1][2];
+  for (int i = lane; i < C::NAB * C::NCD; i += 32) V[i] = 0.0;
+  for (int kl = k0; kl < k1; ++kl) {
+    double q, Qx, Qy, Qz;
+    load_pdat(ket.pdat, kl, q, Qx, Qy, Qz);
+    const double* __restrict__ Ek = ket.Eket + (size_t)kl * (C::NHCD * C::NCD);
+    // single row chunk: stream the bra primitives through one R row, GEMM2 once per ket primitive
+    constexpr bool STREAM = C::NCHUNK == 1 && KR == 1;
+    double t1s[C::MC][C::NT1][2];
+    if constexpr (STREAM) {
 #pragma unroll
       for (int mc = 0; mc < C::MC; ++mc)
 #pragma unroll
-        for (int nt = 0; nt < C::NT1; ++nt) t1[mc][nt][0] = t1[mc][nt][1] = 0.0;
-      for (int ij = b0; ij < b1; ++ij) {
+        for (int nt = 0; nt < C::NT1; ++nt) t1s[mc][nt][0] = t1s[mc][nt][1] = 0.0;
+    }
+    for (int ig0 = b0; ig0 < b1; ig0 += KR) {
+      const int ign = min(KR, b1 - ig0);
+      for (int il = 0; il < ign; ++il) {
         double p, Px, Py, Pz;
-        load_pdat(bra.pdat, ij, p, Px, Py, Pz);
-        compute_R<C>(p, Px, Py, Pz, q, Qx, Qy, Qz, Rbuf, rtab, btab, lane);
-        const double* __restrict__ E = bra.Ebra + (size_t)ij * (C::NAB * C::NHAB);
+        load_pdat(bra.pdat, ig0 + il, p, Px, Py, Pz);
+        compute_R<C>(p, Px, Py, Pz, q, Qx, Qy, Qz, Rbuf + il * NH, Rbuf + KR * NH, rtab, btab, lane);
+      }
+      for (int ch = 0; ch < C::NCHUNK; ++ch) {
+        double t1[C::MC][C::NT1][2];
 #pragma unroll
-        for (int ks = 0; ks < C::KS1; ++ks) {
-          const int pc = 4 * ks + t;
-          double a[C::MC];
-#pragma unroll
-          for (int mc = 0; mc < C::MC; ++mc) {
-            const int row = 8 * (ch * C::MC + mc) + g;
-            a[mc] = (row < C::NAB && pc < C::NHAB) ? __ldg(E + row * C::NHAB + pc) : 0.0;
-          }
+        for (int mc = 0; mc < C::MC; ++mc)
 #pragma unroll
           for (int nt = 0; nt < C::NT1; ++nt) {
-            const int qc = 8 * nt + g;
-            const double b = (pc < C::NHAB && qc < C::NHCD) ? Rbuf[htab[pc * C::NHCD + qc]] : 0.0;
+            t1[mc][nt][0] = STREAM ? t1s[mc][nt][0] : 0.0;
+            t1[mc][nt][1] = STREAM ? t1s[mc][nt][1] : 0.0;
+          }
+        for (int il = 0; il < ign; ++il) {
+          const double* __restrict__ E = bra.Ebra + (size_t)(ig0 + il) * (C::NAB * C::NHAB);
+          const double* __restrict__ Rr = Rbuf + il * NH;
 #pragma unroll
-            for (int mc = 0; mc < C::MC; ++mc)
-              if (ch * C::MC + mc < C::MT) dmma884(t1[mc][nt][0], t1[mc][nt][1], a[mc], b);
+          for (int ks = 0; ks < C::KS1; ++ks) {
+            const int pc = 4 * ks + t;
+            double a[C::MC];
+#pragma unroll
+            for (int mc = 0; mc < C::MC; ++mc) {
+              const int row = 8 * (ch * C::MC + mc) + g;
+              a[mc] = (row < C::NAB && pc < C::NHAB) ? __ldg(E + row * C::NHAB + pc) : 0.0;
+            }
+#pragma unroll
+            for (int nt = 0; nt < C::NT1; ++nt) {
+              const int qc = 8 * nt + g;
+              const double b = (pc < C::NHAB && qc < C::NHCD) ? Rr[htab[pc * C::NHCD + qc]] : 0.0;
+#pragma unroll
+              for (int mc = 0; mc < C::MC; ++mc)
+                if (ch * C::MC + mc < C::MT) dmma884(t1[mc][nt][0], t1[mc][nt][1], a[mc], b);
+            }
           }
         }
-        __syncwarp();
+        if constexpr (STREAM) {
+          // keep accumulating over the next bra primitives; GEMM2 after the last one
+#pragma unroll
+          for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+            for (int nt = 0; nt < C::NT1; ++nt) {
+              t1s[mc][nt][0] = t1[mc][nt][0];
+              t1s[mc][nt][1] = t1[mc][nt][1];
+            }
+          if (ig0 + KR < b1) continue;
+        }
+        // GEMM2: k-step (nt, e) takes q = 8 nt + 2 t + e from the GEMM1 accumulator of lane (g, t)
+        double c2[C::MC][C::NT2][2];
+#pragma unroll
+        for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+          for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
+#pragma unroll
+        for (int nt = 0; nt < C::NT1; ++nt)
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int qq = 8 * nt + 2 * t + e;
+#pragma unroll
+            for (int n2 = 0; n2 < C::NT2; ++n2) {
+              const int cd = 8 * n2 + g;
+              const double b = (qq < C::NHCD && cd < C::NCD) ? __ldg(Ek + qq * C::NCD + cd) : 0.0;
+#pragma unroll
+              for (int mc = 0; mc < C::MC; ++mc)
+                if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
+            }
+          }
+#pragma unroll
+        for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+          for (int n2 = 0; n2 < C::NT2; ++n2)
+#pragma unroll
+            for (int i = 0; i < 2; ++i) {
+              const int row = 8 * (ch * C::MC + mc) + g, col = 8 * n2 + 2 * t + i;
+              if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] += c2[mc][n2][i];
+            }
       }
-      // GEMM2: k-step (nt, e) takes q = 8 nt + 2 t + e from the GEMM1 accumulator of lane (g, t)
-      const double* __restrict__ Ek = ket.Eket + (size_t)kl * (C::NHCD * C::NCD);
-#pragma unroll
-      for (int nt = 0; nt < C::NT1; ++nt)
-#pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          const int qq = 8 * nt + 2 * t + e;
-#pragma unroll
-          for (int n2 = 0; n2 < C::NT2; ++n2) {
-            const int cd = 8 * n2 + g;
-            const double b = (qq < C::NHCD && cd < C::NCD) ? __ldg(Ek + qq * C::NCD + cd) : 0.0;
-#pragma unroll
-            for (int mc = 0; mc < C::MC; ++mc)
-              if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
-          }
-        }
+      __syncwarp();  // R rows are overwritten by the next bra-primitive group
     }
-#pragma unroll
-    for (int mc = 0; mc < C::MC; ++mc)
-#pragma unroll
-      for (int n2 = 0; n2 < C::NT2; ++n2)
-#pragma unroll
-        for (int i = 0; i < 2; ++i) {
-          const int row = 8 * (ch * C::MC + mc) + g, col = 8 * n2 + 2 * t + i;
-          if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] = c2[mc][n2][i];
-        }
   }
   __syncwarp();
 }
