@@ -47,7 +47,9 @@ struct SlabCfg {
 
 template <int X, int Y>
 constexpr bool use_slab() {
-  return !use_tpq(X, Y) && SlabCfg<X, Y>::OK;
+  // measured per class (profiles/README.md): only (pp|pp) and (dp|pp) -- bras with up to 16 primitive
+  // pairs and pp kets -- still beat the warp-per-quartet kernel with its once-per-quartet R rows
+  return !use_tpq(X, Y) && SlabCfg<X, Y>::OK && ((X == 2 && Y == 2) || (X == 4 && Y == 2));
 }
 
 template <int X, int Y>
