@@ -71,29 +71,39 @@ def workload_flops(sh, Q, tau, prim_eps=PRIM_EPS):
                 continue
             buckets.setdefault(la * (la + 1) // 2 + lb, []).append((Q[a, b], K))
     qmax = max(q for v in buckets.values() for q, _ in v)
+    # library order: primitive-count group, then Q descending (csrc/mako_internal.h kgroup)
+    def kgroup(K):
+        return K - 1 if K <= 4 else (4 if K <= 6 else 5 if K <= 9 else 6 if K <= 12 else 7 if K <= 16 else
+                                     8 if K <= 24 else 9 if K <= 36 else 10)
     for k in list(buckets):
-        v = sorted([x for x in buckets[k] if x[0] * qmax >= tau], key=lambda x: -x[0])
-        buckets[k] = (np.array([x[0] for x in v]), np.array([x[1] for x in v], np.int64))
+        v = sorted([x for x in buckets[k] if x[0] * qmax >= tau], key=lambda x: (kgroup(x[1]), -x[0]))
+        buckets[k] = (np.array([x[0] for x in v]), np.array([x[1] for x in v], np.int64),
+                      np.array([kgroup(x[1]) for x in v], np.int64))
     bl = lambda b: [(0, 0), (1, 0), (1, 1), (2, 0), (2, 1), (2, 2), (3, 0), (3, 1), (3, 2), (3, 3)][b]
     total, nq = 0.0, 0
     for X in buckets:
         for Y in buckets:
             if Y > X:
                 continue
-            QX, KX = buckets[X]
-            QY, KY = buckets[Y]
+            QX, KX, GX = buckets[X]
+            QY, KY, GY = buckets[Y]
             la, lb = bl(X)
             lc, ld = bl(Y)
             nab, ncd = (2 * la + 1) * (2 * lb + 1), (2 * lc + 1) * (2 * ld + 1)
             hab, hcd = _nH(la + lb), _nH(lc + ld)
             cK = np.concatenate([[0], np.cumsum(KY)])
-            # kets with QP * QY >= tau: prefix of descending QY
-            cnt = np.array([np.searchsorted(-(qp * QY), -tau, side="right") for qp in QX], np.int64)
-            if X == Y:
-                cnt = np.minimum(cnt, np.arange(1, len(QX) + 1))
-            sK = cK[cnt]
-            total += float(np.sum(KX * sK) * 2.0 * nab * hab * hcd + np.sum(sK) * 2.0 * nab * hcd * ncd)
-            nq += int(cnt.sum())
+            for g in range(11):
+                s0, s1 = np.searchsorted(GY, g, "left"), np.searchsorted(GY, g, "right")
+                if s1 <= s0:
+                    continue
+                seg = QY[s0:s1]
+                # kets of the group with QP * Q >= tau: prefix of the descending segment
+                cnt = np.array([np.searchsorted(-(qp * seg), -tau, side="right") for qp in QX], np.int64)
+                if X == Y:  # canonical: ket position <= bra position
+                    cnt = np.minimum(cnt, np.maximum(0, np.arange(len(QX)) - s0 + 1))
+                sK = cK[s0 + cnt] - cK[s0]
+                total += float(np.sum(KX * sK) * 2.0 * nab * hab * hcd + np.sum(sK) * 2.0 * nab * hcd * ncd)
+                nq += int(cnt.sum())
     return total, nq
 
 
@@ -153,13 +163,14 @@ def cpu_baseline(sh, D, tau, total_flops, target_s=15.0, Q=None):
     import oracle
     if Q is None:
         Q = oracle.schwarz(sh)
-    # pilot on a tiny shard, then size the sample to ~target_s
+    # pilot on 8 spread-out tiny shards, then size the sample to ~target_s
     npair = sh.nshell * (sh.nshell + 1) // 2
-    S = max(2, min(npair, 50000))
+    S = max(2, min(npair, 20000))
     t0 = time.perf_counter()
-    oracle.jk(sh, D, tau, 1, S, Q=Q)
-    tp = time.perf_counter() - t0
-    est_total = max(tp, 1e-3) * S
+    for i in range(8):
+        oracle.jk(sh, D, tau, (i * S) // 8 + 1, S, Q=Q)
+    tp = (time.perf_counter() - t0) / 8
+    est_total = max(tp, 1e-4) * S
     S = int(min(max(2, est_total / target_s), npair))
     shard = S // 2
     t0 = time.perf_counter()

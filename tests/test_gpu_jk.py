@@ -140,3 +140,14 @@ def test_valinomycin_full_size_sampled_blocks():
         print("valinomycin block", x, y, np.abs(jb).max(), np.abs(kb).max(), np.abs(gj - jb).max(), np.abs(gk - kb).max())
         assert np.abs(jb).max() > 1e-3 and np.abs(kb).max() > 1e-6
         assert np.abs(gj - jb).max() <= 1e-8 and np.abs(gk - kb).max() <= 1e-8
+
+
+def test_flop_accounting_library_equals_reference_arm():
+    """bench.py's reference arm counts the workload's algorithmic FLOPs in Python from the oracle's Q;
+    the library counts them from its own pair data: both must agree (same screening, same order)."""
+    import bench
+    m, sh, B, P = _setup("benzene-def2svp", 1e-12)
+    lib = P.flops()
+    py_flops, py_q = bench.workload_flops(sh, oracle.schwarz(sh), 1e-12)
+    assert py_q == lib["quartets"]
+    assert abs(py_flops - lib["gemm_flops"]) <= 1e-9 * lib["gemm_flops"]
