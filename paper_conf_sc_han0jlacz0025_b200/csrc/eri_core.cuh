@@ -97,6 +97,11 @@ __device__ void init_tables(uint16_t* htab, uint32_t* rtab) {
   }
 }
 
+// 256-bit read-only global load (sm_100a LDG.E.ENL2.256): 4 doubles from a 32 B aligned address
+__device__ __forceinline__ void ldg256(const double* __restrict__ p, double& a, double& b, double& c, double& d) {
+  asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+}
+
 // 1/sqrt(x) for positive normal x: float seed + two Newton steps (no slow path)
 __device__ __forceinline__ double rsqrt_fast(double x) {
   double y = (double)rsqrtf((float)x);
@@ -112,13 +117,22 @@ __device__ __forceinline__ double rsqrt_fast(double x) {
 //           recursion F_m = (2T F_{m+1} + e^{-T}) / (2m+1).
 //  T >= 40: F_0 = (1/2) sqrt(pi/T) (erfc(sqrt 40) < 1e-18), upward F_{m+1} = ((2m+1)F_m - e^{-T})/(2T)
 //           with exp(-T) from a second 1/32 grid for T < 80 and dropped beyond (< 1e-18 relative).
-template <int L>
+// WIDE: 256-bit row loads (lane-private lookups, per-lane kernels); otherwise 128-bit loads (the
+// warp-uniform lookups of the warp-cooperative R, measured faster with the narrower form)
+template <int L, bool WIDE = false>
 __device__ __forceinline__ void boys_eval(double T, const double* __restrict__ tab, double (&F)[L + 1]) {
   if (T < BOYS_TMAX) {
     const int k = __double2int_rn(T * (1.0 / BOYS_H));
     const double x = fma((double)k, BOYS_H, -T);
-    const double2* r = reinterpret_cast<const double2*>(tab + ((size_t)L * BOYS_NGRID + k) * BOYS_ROW);
-    const double2 r01 = __ldg(r), r23 = __ldg(r + 1), r45 = __ldg(r + 2), r6e = __ldg(r + 3);
+    const double* r = tab + ((size_t)L * BOYS_NGRID + k) * BOYS_ROW;  // 64 B row
+    double2 r01, r23, r45, r6e;
+    if constexpr (WIDE) {
+      ldg256(r, r01.x, r01.y, r23.x, r23.y);
+      ldg256(r + 4, r45.x, r45.y, r6e.x, r6e.y);
+    } else {
+      const double2* r2 = reinterpret_cast<const double2*>(r);
+      r01 = __ldg(r2); r23 = __ldg(r2 + 1); r45 = __ldg(r2 + 2); r6e = __ldg(r2 + 3);
+    }
     const double x2 = x * 0.5, x3 = x * (1.0 / 3.0), x4 = x * 0.25, x5 = x * 0.2, x6 = x * (1.0 / 6.0);
     double f = r6e.x;
     f = fma(f, x6, r45.y);
@@ -214,12 +228,17 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
   }
 }
 
-// primitive-pair record {p, Px, Py, Pz} (32 B aligned): two 128-bit loads
+// primitive-pair record {p, Px, Py, Pz} (32 B aligned): one 256-bit load (WIDE) or two 128-bit loads
+template <bool WIDE = false>
 __device__ __forceinline__ void load_pdat(const double* __restrict__ pdat, int i, double& p, double& x, double& y,
                                           double& z) {
-  const double2* v = reinterpret_cast<const double2*>(pdat + 4 * (size_t)i);
-  const double2 a = __ldg(v), b = __ldg(v + 1);
-  p = a.x; x = a.y; y = b.x; z = b.y;
+  if constexpr (WIDE) {
+    ldg256(pdat + 4 * (size_t)i, p, x, y, z);
+  } else {
+    const double2* v = reinterpret_cast<const double2*>(pdat + 4 * (size_t)i);
+    const double2 a = __ldg(v), b = __ldg(v + 1);
+    p = a.x; x = a.y; y = b.x; z = b.y;
+  }
 }
 
 __device__ __forceinline__ void dmma884(double& c0, double& c1, double a, double b) {

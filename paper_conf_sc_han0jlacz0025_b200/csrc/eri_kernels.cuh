@@ -36,9 +36,28 @@ __host__ __device__ constexpr size_t cta_smem_bytes() {
   return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)CTA_WARPS * C::WARP_DBL;
 }
 
-// Persistent J/K kernel: each warp pulls tasks (bra pair, <= KT consecutive kets) from a global counter.
+// occupancy cap (4 CTAs/SM, <= 128 registers) measured faster for the fd-bra classes and (fp|dd) only
 template <int X, int Y>
-__global__ void __launch_bounds__(CTA_THREADS) jk_kernel(JKArgs a) {
+constexpr int jk_minb() {
+  return (X == 8 || (X == 7 && Y == 5)) ? 4 : 1;
+}
+
+// Persistent J/K kernel: each warp pulls tasks (bra pair, <= KT consecutive kets) from a global counter.
+// (An explicit minBlocks of 1 changes ptxas' register heuristic, so the cap is a separate wrapper.)
+template <int X, int Y>
+__device__ __forceinline__ void jk_body(const JKArgs& a);
+template <int X, int Y>
+__global__ void __launch_bounds__(CTA_THREADS) jk_kernel_free(JKArgs a) { jk_body<X, Y>(a); }
+template <int X, int Y>
+__global__ void __launch_bounds__(CTA_THREADS, 4) jk_kernel_capped(JKArgs a) { jk_body<X, Y>(a); }
+template <int X, int Y>
+constexpr auto jk_kernel_ptr() {
+  if constexpr (jk_minb<X, Y>() > 1) return &jk_kernel_capped<X, Y>;
+  else return &jk_kernel_free<X, Y>;
+}
+
+template <int X, int Y>
+__device__ __forceinline__ void jk_body(const JKArgs& a) {
   using C = ClsXY<X, Y>;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   uint16_t* htab = reinterpret_cast<uint16_t*>(smem_raw);
@@ -151,12 +170,12 @@ int jk_blocks_per_sm() {
     int nb = 0;
     if constexpr (use_kf_swap<X, Y>()) {
       constexpr size_t ks = KfCfg<Y, X>::SMEM;
-      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel<Y, X>, ks)) return 1;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel<Y, X>, CTA_THREADS, ks);
+      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel_ptr<Y, X>(), ks)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel_ptr<Y, X>(), CTA_THREADS, ks);
     } else if constexpr (use_kf<X, Y>()) {
       constexpr size_t ks = KfCfg<X, Y>::SMEM;
-      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel<X, Y>, ks)) return 1;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel<X, Y>, CTA_THREADS, ks);
+      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel_ptr<X, Y>(), ks)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel_ptr<X, Y>(), CTA_THREADS, ks);
     } else if constexpr (use_tpq(X, Y)) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, tpq_jk_kernel<X, Y>, CTA_THREADS, 0);
     } else if constexpr (use_slab<X, Y>()) {
@@ -164,8 +183,8 @@ int jk_blocks_per_sm() {
       if (set_smem_attr<X, Y>((const void*)slab_jk_kernel<X, Y>, ss)) return 1;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, slab_jk_kernel<X, Y>, CTA_THREADS, ss);
     } else {
-      if (set_smem_attr<X, Y>((const void*)jk_kernel<X, Y>, smem)) return 1;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel<X, Y>, CTA_THREADS, smem);
+      if (set_smem_attr<X, Y>((const void*)jk_kernel_ptr<X, Y>(), smem)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel_ptr<X, Y>(), CTA_THREADS, smem);
     }
     cached = nb < 1 ? 1 : nb;
   }
@@ -187,15 +206,15 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   if (cap < nsm) cap = nsm;
   const int grid = (int)(want < cap ? want : cap);
   if constexpr (use_kf_swap<X, Y>())
-    kf_jk_kernel<Y, X><<<grid, CTA_THREADS, KfCfg<Y, X>::SMEM, (cudaStream_t)stream>>>(a);
+    kf_jk_kernel_ptr<Y, X>()<<<grid, CTA_THREADS, KfCfg<Y, X>::SMEM, (cudaStream_t)stream>>>(a);
   else if constexpr (use_kf<X, Y>())
-    kf_jk_kernel<X, Y><<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
+    kf_jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
   else if constexpr (use_tpq(X, Y))
     tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, (cudaStream_t)stream>>>(a);
   else if constexpr (use_slab<X, Y>())
     slab_jk_kernel<X, Y><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
   else
-    jk_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
+    jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("jk_kernel launch: ") + cudaGetErrorString(e));
   if (nlaunch) ++*nlaunch;

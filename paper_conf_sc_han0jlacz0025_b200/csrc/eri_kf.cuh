@@ -65,7 +65,19 @@ constexpr bool use_kf_swap() {
 }
 
 template <int X, int Y>
-__global__ void __launch_bounds__(128, KfCfg<X, Y>::MINB) kf_jk_kernel(JKArgs a) {
+__device__ __forceinline__ void kf_body(const JKArgs& a);
+template <int X, int Y>
+__global__ void __launch_bounds__(128) kf_kernel_free(JKArgs a) { kf_body<X, Y>(a); }
+template <int X, int Y>
+__global__ void __launch_bounds__(128, 3) kf_kernel_capped(JKArgs a) { kf_body<X, Y>(a); }
+template <int X, int Y>
+constexpr auto kf_jk_kernel_ptr() {
+  if constexpr (KfCfg<X, Y>::MINB > 1) return &kf_kernel_capped<X, Y>;
+  else return &kf_kernel_free<X, Y>;
+}
+
+template <int X, int Y>
+__device__ __forceinline__ void kf_body(const JKArgs& a) {
   using C = ClsXY<X, Y>;
   using K = KfCfg<X, Y>;
   constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
@@ -114,7 +126,7 @@ __global__ void __launch_bounds__(128, KfCfg<X, Y>::MINB) kf_jk_kernel(JKArgs a)
         for (int j = 0; j < NCD; ++j) W[i][j] = 0.0;
       for (int kl = k0; kl < k1; ++kl) {
         double q, Qx, Qy, Qz;
-        load_pdat(a.ket.pdat, kl, q, Qx, Qy, Qz);
+        load_pdat<true>(a.ket.pdat, kl, q, Qx, Qy, Qz);
         double Rr[nH(L)];
         r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
         const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);

@@ -156,7 +156,7 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
           double p, Px, Py, Pz;
         load_pdat(a.bra.pdat, ij, p, Px, Py, Pz);
           double q, Qx, Qy, Qz;
-        load_pdat(a.ket.pdat, klc, q, Qx, Qy, Qz);
+        load_pdat<true>(a.ket.pdat, klc, q, Qx, Qy, Qz);
           double Rr[nH(L)];
           r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
           double* row = Rs + (size_t)c * RS;

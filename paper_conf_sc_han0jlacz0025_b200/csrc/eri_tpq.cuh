@@ -47,7 +47,17 @@ __device__ __forceinline__ void static_for(F&& f) {
 // NH x NC doubles (contiguous, 16 B aligned when NH*NC is even) into a register matrix
 template <int NH, int NC>
 __device__ __forceinline__ void load_mat(const double* __restrict__ src, double (&M)[NH][NC]) {
-  if constexpr ((NH * NC) % 2 == 0) {
+  if constexpr ((NH * NC) % 4 == 0) {  // 32 B aligned rows of the E~ array: 256-bit loads
+    static_for<0, NH * NC / 4>([&](auto ic) {
+      constexpr int i = decltype(ic)::value;
+      double w0, w1, w2, w3;
+      ldg256(src + 4 * i, w0, w1, w2, w3);
+      M[(4 * i) / NC][(4 * i) % NC] = w0;
+      M[(4 * i + 1) / NC][(4 * i + 1) % NC] = w1;
+      M[(4 * i + 2) / NC][(4 * i + 2) % NC] = w2;
+      M[(4 * i + 3) / NC][(4 * i + 3) % NC] = w3;
+    });
+  } else if constexpr ((NH * NC) % 2 == 0) {
     const double2* v = reinterpret_cast<const double2*>(src);
     static_for<0, NH * NC / 2>([&](auto ic) {
       constexpr int i = decltype(ic)::value;
@@ -96,7 +106,7 @@ __device__ __forceinline__ void r_regs(double p, double Px, double Py, double Pz
   const double pq = p + q, ri = rsqrt_fast(pq), rho = p * q * ri * ri;
   const double X = Px - Qx, Y = Py - Qy, Z = Pz - Qz;
   double F[L + 1];
-  boys_eval<L>(rho * (X * X + Y * Y + Z * Z), btab, F);
+  boys_eval<L, true>(rho * (X * X + Y * Y + Z * Z), btab, F);
   double s = TWO_PI_52 * ri;
   const double m2r = -2.0 * rho;
 #pragma unroll
@@ -174,7 +184,7 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
             for (int j = 0; j < NCD; ++j) W[h][j] = 0.0;
           for (int kl = k0; kl < k1; ++kl) {
             double q, Qx, Qy, Qz;
-        load_pdat(a.ket.pdat, kl, q, Qx, Qy, Qz);
+        load_pdat<true>(a.ket.pdat, kl, q, Qx, Qy, Qz);
             double Ek[NHCD][NCD];
             const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
             load_mat<NHCD, NCD>(ek, Ek);
@@ -203,7 +213,7 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
       } else {
       for (int kl = k0; kl < k1; ++kl) {
         double q, Qx, Qy, Qz;
-        load_pdat(a.ket.pdat, kl, q, Qx, Qy, Qz);
+        load_pdat<true>(a.ket.pdat, kl, q, Qx, Qy, Qz);
         // signed ket E~^T [q][cd]
         double Ek[NHCD][NCD];
         const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
