@@ -115,6 +115,20 @@ void mako_pairs_destroy(mako_pairs pairs);
 mako_status mako_build_jk(mako_pairs pairs, const double* D, double thresh, double* J, double* K, int shard,
                           int nshards, void* cuda_stream);
 
+/* Density-weighted screening (S3.2.3 "density-weighted Schwarz ... pruned"; SURVEY
+ * S8.f row 2; reading R17).  With flags = MAKO_JK_DENSITY_SCREEN, mako_build_jk_ex keeps a
+ * canonical quartet only if, in addition to Q_ab Q_cd >= the pairs' threshold,
+ *     Q_ab Q_cd Dmax(ab,cd) >= thresh,
+ * Dmax(ab,cd) = the largest max|D_mn| over the six shell blocks (ab)(cd)(ac)(ad)(bc)(bd) the quartet
+ * is contracted with.  A dropped quartet changes no J or K element by more than 2*thresh (its
+ * |(mn|ls)| <= Q_ab Q_cd by Cauchy-Schwarz, and each of its J/K updates is (degeneracy <= 1) x 2 x
+ * |(mn|ls) D|).  Intended for incremental SCF builds (D = Delta D).  This mode computes the block
+ * maxima on the device and SYNCHRONISES cuda_stream once (the task plan depends on max|D|);
+ * otherwise identical to mako_build_jk (flags = 0 is exactly mako_build_jk). */
+#define MAKO_JK_DENSITY_SCREEN 1u
+mako_status mako_build_jk_ex(mako_pairs pairs, const double* D, double thresh, unsigned flags, double* J, double* K,
+                             int shard, int nshards, void* cuda_stream);
+
 /* Number of CUDA kernels one mako_build_jk call launches for these arguments (for bench accounting). */
 mako_status mako_build_jk_launches(mako_pairs pairs, double thresh, int shard, int nshards, int* n_launches);
 

@@ -8,6 +8,9 @@ import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libmako.so")
+# experiments only: MAKO_LIB names an alternative in-tree build (build.py --variant NAME -> libmako_NAME.so)
+if os.environ.get("MAKO_LIB"):
+    LIB_PATH = os.path.join(HERE, "libmako_%s.so" % os.environ["MAKO_LIB"])
 
 MAKO_OK = 0
 NCLASS = 55
@@ -18,7 +21,7 @@ STATUS = {0: "MAKO_OK", 1: "MAKO_ERR_INVALID", 2: "MAKO_ERR_UNSUPPORTED", 3: "MA
 EXPORTS = ["mako_basis_create", "mako_basis_nbf", "mako_basis_nshell", "mako_basis_ao_offsets", "mako_basis_destroy",
            "mako_shellpairs_screen", "mako_pairs_stats", "mako_pairs_flops", "mako_pairs_destroy", "mako_build_jk",
            "mako_build_jk_launches", "mako_eri_batch", "mako_boys", "mako_last_error", "mako_version",
-           "mako_pairs_class_flops", "mako_profile_enable", "mako_profile_read"]
+           "mako_pairs_class_flops", "mako_profile_enable", "mako_profile_read", "mako_build_jk_ex"]
 
 
 class MakoError(RuntimeError):
@@ -56,6 +59,8 @@ def load():
                               ctypes.POINTER(_ll)], ctypes.c_int),
         "mako_pairs_destroy": ([_vp], None),
         "mako_build_jk": ([_vp, _vp, ctypes.c_double, _vp, _vp, ctypes.c_int, ctypes.c_int, _vp], ctypes.c_int),
+        "mako_build_jk_ex": ([_vp, _vp, ctypes.c_double, ctypes.c_uint, _vp, _vp, ctypes.c_int, ctypes.c_int, _vp],
+                             ctypes.c_int),
         "mako_build_jk_launches": ([_vp, ctypes.c_double, ctypes.c_int, ctypes.c_int, _ip], ctypes.c_int),
         "mako_eri_batch": ([_vp, ctypes.c_int, _ip, _vp, ctypes.c_size_t, _vp], ctypes.c_int),
         "mako_boys": ([ctypes.c_int, _vp, ctypes.c_int, _vp, _vp], ctypes.c_int),

@@ -47,7 +47,8 @@ struct Cls {
   // R rows kept per bra primitive (computed once per primitive quartet, reused by every row chunk)
   // (d/f x d/f bra pairs are single-primitive in the def2/cc families: no rows to group)
   static constexpr int KR = (LA >= 2 && LB >= 2) ? 1 : clampi(1200 / NH - 1, 1, 4);
-  static constexpr int W_R = (KR + 1) * NH;  // KR result rows + 1 ping-pong scratch row
+  // KR result rows + 1 ping-pong scratch row; doubles as the digestion partial-sum scratch (Ps)
+  static constexpr int W_R = ((KR + 1) * NH > 2 * (NA + NB) * NCD) ? (KR + 1) * NH : 2 * (NA + NB) * NCD;
   static constexpr int W_V = NAB * NCD; // (ab|cd) block
   static constexpr int W_J = NAB;       // J_ab partial sums over the kets of a task
   static constexpr int W_D = NA * NB + NC * ND + NA * NC + NA * ND + NB * NC + NB * ND;  // staged D blocks
@@ -101,6 +102,14 @@ __device__ void init_tables(uint16_t* htab, uint32_t* rtab) {
 __device__ __forceinline__ void ldg256(const double* __restrict__ p, double& a, double& b, double& c, double& d) {
   asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
 }
+
+// asynchronous 8-byte global -> shared copy (LDGSTS, no register staging) and its completion wait
+__device__ __forceinline__ void cp_async8(double* smem_dst, const double* gsrc) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
 // 1/sqrt(x) for positive normal x: float seed + two Newton steps (no slow path)
 __device__ __forceinline__ double rsqrt_fast(double x) {
@@ -257,15 +266,24 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
                               double* __restrict__ V, const uint16_t* __restrict__ htab,
                               const uint32_t* __restrict__ rtab, const double* __restrict__ btab, int lane) {
   constexpr int KR = C::KR, NH = C::NH;
+  // one row chunk with small accumulators: the GEMM2 accumulators stay in registers across all
+  // primitive quartets and V is written once; otherwise each chunk adds its rows into V (SMEM)
+  constexpr bool ONECHUNK = C::NCHUNK == 1 && 2 * C::MC * (C::NT1 + C::NT2) <= 24;
   const int g = lane >> 2, t = lane & 3;
   const int b0 = __ldg(bra.poff + P), b1 = __ldg(bra.poff + P + 1);
   const int k0 = __ldg(ket.poff + R), k1 = __ldg(ket.poff + R + 1);
-  for (int i = lane; i < C::NAB * C::NCD; i += 32) V[i] = 0.0;
+  if constexpr (!ONECHUNK)
+    for (int i = lane; i < C::NAB * C::NCD; i += 32) V[i] = 0.0;
+  double c2[C::MC][C::NT2][2];
+#pragma unroll
+  for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+    for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
   for (int kl = k0; kl < k1; ++kl) {
     double q, Qx, Qy, Qz;
     load_pdat(ket.pdat, kl, q, Qx, Qy, Qz);
     const double* __restrict__ Ek = ket.Eket + (size_t)kl * (C::NHCD * C::NCD);
-    // single row chunk: stream the bra primitives through one R row, GEMM2 once per ket primitive
+    // single row chunk and one R row: stream the bra primitives through it, GEMM2 once per ket primitive
     constexpr bool STREAM = C::NCHUNK == 1 && KR == 1;
     double t1s[C::MC][C::NT1][2];
     if constexpr (STREAM) {
@@ -323,12 +341,13 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
             }
           if (ig0 + KR < b1) continue;
         }
+        if constexpr (!ONECHUNK) {
+#pragma unroll
+          for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+            for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
+        }
         // GEMM2: k-step (nt, e) takes q = 8 nt + 2 t + e from the GEMM1 accumulator of lane (g, t)
-        double c2[C::MC][C::NT2][2];
-#pragma unroll
-        for (int mc = 0; mc < C::MC; ++mc)
-#pragma unroll
-          for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
 #pragma unroll
         for (int nt = 0; nt < C::NT1; ++nt)
 #pragma unroll
@@ -343,18 +362,31 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
                 if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
             }
           }
+        if constexpr (!ONECHUNK) {
 #pragma unroll
-        for (int mc = 0; mc < C::MC; ++mc)
+          for (int mc = 0; mc < C::MC; ++mc)
 #pragma unroll
-          for (int n2 = 0; n2 < C::NT2; ++n2)
+            for (int n2 = 0; n2 < C::NT2; ++n2)
 #pragma unroll
-            for (int i = 0; i < 2; ++i) {
-              const int row = 8 * (ch * C::MC + mc) + g, col = 8 * n2 + 2 * t + i;
-              if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] += c2[mc][n2][i];
-            }
+              for (int i = 0; i < 2; ++i) {
+                const int row = 8 * (ch * C::MC + mc) + g, col = 8 * n2 + 2 * t + i;
+                if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] += c2[mc][n2][i];
+              }
+        }
       }
       __syncwarp();  // R rows are overwritten by the next bra-primitive group
     }
+  }
+  if constexpr (ONECHUNK) {
+#pragma unroll
+    for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+      for (int n2 = 0; n2 < C::NT2; ++n2)
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int row = 8 * mc + g, col = 8 * n2 + 2 * t + i;
+          if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] = c2[mc][n2][i];
+        }
   }
   __syncwarp();
 }
@@ -363,40 +395,65 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
 // With v' = deg * (ab|cd), deg = 1/2 per coincidence (a=b, c=d, ab=cd), the 8 permutations of a
 // canonical quartet reduce for symmetric D to the 6 forward updates below; the transposed halves
 // are restored by J = Jacc + Jacc^T, K = Kacc + Kacc^T at the end of the build.
-// The six D sub-blocks are first staged in warp SMEM (Ds, DIGEST_DS doubles) with coalesced row
-// loads, so the reduction loops below run on SMEM with two independent accumulators.
+// V is the warp-SMEM block V[ab][cd] (row stride NCD).  Steps:
+//   1. the six D sub-blocks are staged in warp SMEM (Ds) with coalesced row loads;
+//   2. J_ab: row pass (lane = ab), accumulated in SMEM over the kets of a task;
+//   3. one column pass (lane = cd = (c,d)) reads every V element ONCE and forms, in registers,
+//        K_ac partial  sum_b v D_bd   (per a)      K_ad partial  sum_b v D_bc   (per a)
+//        K_bc partial  sum_a v D_ad   (per b)      K_bd partial  sum_a v D_ac   (per b)
+//        J_cd          sum_ab v D_ab  (complete per lane)
+//      the K partials go to SMEM (Ps) as [a or b][cd];
+//   4. K_ac/K_bc sum their partials over d, K_ad/K_bd over c, one FP64 atomic per K element.
 template <class C>
 struct DigestLayout {
   static constexpr int AB = 0, CD = AB + C::NA * C::NB, AC = CD + C::NC * C::ND, AD = AC + C::NA * C::NC,
                        BC = AD + C::NA * C::ND, BD = BC + C::NB * C::NC, TOT = BD + C::NB * C::ND;
+  // partial sums (Ps): [NA][NCD] x 2, [NB][NCD] x 2
+  static constexpr int PAC = 0, PAD = PAC + C::NA * C::NCD, PBC = PAD + C::NA * C::NCD, PBD = PBC + C::NB * C::NCD,
+                       PTOT = PBD + C::NB * C::NCD;
 };
-constexpr int DIGEST_DS = 6 * 49;
 
+// offset in D of staged element x (D_ab | D_cd | D_ac | D_ad | D_bc | D_bd)
 template <class C>
+__device__ __forceinline__ size_t d_offset(int x, int oa, int ob, int oc, int od, int nbf) {
+  using DL = DigestLayout<C>;
+  constexpr int NB = C::NB, NC = C::NC, ND = C::ND;
+  int r, c;
+  if (x < DL::CD) { r = oa + (x - DL::AB) / NB; c = ob + (x - DL::AB) % NB; }
+  else if (x < DL::AC) { r = oc + (x - DL::CD) / ND; c = od + (x - DL::CD) % ND; }
+  else if (x < DL::AD) { r = oa + (x - DL::AC) / NC; c = oc + (x - DL::AC) % NC; }
+  else if (x < DL::BC) { r = oa + (x - DL::AD) / ND; c = od + (x - DL::AD) % ND; }
+  else if (x < DL::BD) { r = ob + (x - DL::BC) / NC; c = oc + (x - DL::BC) % NC; }
+  else { r = ob + (x - DL::BD) / ND; c = od + (x - DL::BD) % ND; }
+  return (size_t)r * nbf + c;
+}
+
+// D sub-blocks of one quartet copied to warp SMEM asynchronously (cp.async), issued before the
+// quartet's ERI work and waited for before its digestion: the L2 latency of the scattered D reads is
+// hidden behind the ERI evaluation
+template <class C>
+__device__ __forceinline__ void d_prefetch(double* __restrict__ Ds, const double* __restrict__ D, int oa, int ob,
+                                           int oc, int od, int nbf, int lane) {
+  for (int x = lane; x < DigestLayout<C>::TOT; x += 32) cp_async8(Ds + x, D + d_offset<C>(x, oa, ob, oc, od, nbf));
+  cp_async_commit();
+}
+
+template <class C, bool STAGE = true>
 __device__ void digest(const double* __restrict__ V, double deg, int oa, int ob, int oc, int od,
                        const double* __restrict__ D, int nbf, double* __restrict__ J, double* __restrict__ K,
-                       double* __restrict__ jab, double* __restrict__ Ds, int lane) {
+                       double* __restrict__ jab, double* __restrict__ Ds, double* __restrict__ Ps, int lane) {
   using DL = DigestLayout<C>;
   constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND, NCD = C::NCD;
-  // stage D_ab, D_cd, D_ac, D_ad, D_bc, D_bd
-  for (int x = lane; x < DL::TOT; x += 32) {
-    int r, c;
-    if (x < DL::CD) { r = oa + (x - DL::AB) / NB; c = ob + (x - DL::AB) % NB; }
-    else if (x < DL::AC) { r = oc + (x - DL::CD) / ND; c = od + (x - DL::CD) % ND; }
-    else if (x < DL::AD) { r = oa + (x - DL::AC) / NC; c = oc + (x - DL::AC) % NC; }
-    else if (x < DL::BC) { r = oa + (x - DL::AD) / ND; c = od + (x - DL::AD) % ND; }
-    else if (x < DL::BD) { r = ob + (x - DL::BC) / NC; c = oc + (x - DL::BC) % NC; }
-    else { r = ob + (x - DL::BD) / ND; c = od + (x - DL::BD) % ND; }
-    Ds[x] = __ldg(D + (size_t)r * nbf + c);
+  // 1. stage D_ab, D_cd, D_ac, D_ad, D_bc, D_bd (unless the caller prefetched them: d_prefetch)
+  if constexpr (STAGE) {
+    for (int x = lane; x < DL::TOT; x += 32) Ds[x] = __ldg(D + d_offset<C>(x, oa, ob, oc, od, nbf));
+  } else {
+    cp_async_wait_all();
   }
   __syncwarp();
   const double* Dab = Ds + DL::AB;
   const double* Dcd = Ds + DL::CD;
-  const double* Dac = Ds + DL::AC;
-  const double* Dad = Ds + DL::AD;
-  const double* Dbc = Ds + DL::BC;
-  const double* Dbd = Ds + DL::BD;
-  // J_ab (accumulated in SMEM across the kets of the task)
+  // 2. J_ab (row pass; odd row stride NCD keeps it bank-conflict free)
   for (int ab = lane; ab < C::NAB; ab += 32) {
     double s0 = 0.0, s1 = 0.0;
     int cd = 0;
@@ -407,61 +464,67 @@ __device__ void digest(const double* __restrict__ V, double deg, int oa, int ob,
     if (cd < NCD) s0 = fma(V[ab * NCD + cd], Dcd[cd], s0);
     jab[ab] = fma(2.0 * deg, s0 + s1, jab[ab]);
   }
-  // J_cd
+  // 3. column pass
   for (int cd = lane; cd < NCD; cd += 32) {
-    double s0 = 0.0, s1 = 0.0;
-    int ab = 0;
-    for (; ab + 1 < C::NAB; ab += 2) {
-      s0 = fma(V[ab * NCD + cd], Dab[ab], s0);
-      s1 = fma(V[(ab + 1) * NCD + cd], Dab[ab + 1], s1);
+    const int c = cd / ND, d = cd % ND;
+    double dbd[NB], dbc[NB], kbc[NB], kbd[NB];
+#pragma unroll
+    for (int b = 0; b < NB; ++b) {
+      dbd[b] = Ds[DL::BD + b * ND + d];
+      dbc[b] = Ds[DL::BC + b * NC + c];
+      kbc[b] = 0.0;
+      kbd[b] = 0.0;
     }
-    if (ab < C::NAB) s0 = fma(V[ab * NCD + cd], Dab[ab], s0);
-    atomicAdd(J + (size_t)(oc + cd / ND) * nbf + od + cd % ND, 2.0 * deg * (s0 + s1));
+    double jcd0 = 0.0, jcd1 = 0.0;
+#pragma unroll
+    for (int a = 0; a < NA; ++a) {
+      const double dad = Ds[DL::AD + a * ND + d], dac = Ds[DL::AC + a * NC + c];
+      double kac = 0.0, kad = 0.0;
+#pragma unroll
+      for (int b = 0; b < NB; ++b) {
+        const double v = V[(a * NB + b) * NCD + cd];
+        kac = fma(v, dbd[b], kac);
+        kad = fma(v, dbc[b], kad);
+        kbc[b] = fma(v, dad, kbc[b]);
+        kbd[b] = fma(v, dac, kbd[b]);
+        if (b & 1) jcd1 = fma(v, Dab[a * NB + b], jcd1); else jcd0 = fma(v, Dab[a * NB + b], jcd0);
+      }
+      Ps[DL::PAC + a * NCD + cd] = kac;
+      Ps[DL::PAD + a * NCD + cd] = kad;
+    }
+#pragma unroll
+    for (int b = 0; b < NB; ++b) {
+      Ps[DL::PBC + b * NCD + cd] = kbc[b];
+      Ps[DL::PBD + b * NCD + cd] = kbd[b];
+    }
+    atomicAdd(J + (size_t)(oc + c) * nbf + od + d, 2.0 * deg * (jcd0 + jcd1));
   }
-  // K_ac += v D_bd | K_ad += v D_bc | K_bc += v D_ad | K_bd += v D_ac   (one flattened index space)
+  __syncwarp();
+  // 4. K_ac[a][c] = sum_d P_ac[a][c,d] | K_ad[a][d] = sum_c P_ad[a][c,d] |
+  //    K_bc[b][c] = sum_d P_bc[b][c,d] | K_bd[b][d] = sum_c P_bd[b][c,d]
   constexpr int N1 = NA * NC, N2 = N1 + NA * ND, N3 = N2 + NB * NC, N4 = N3 + NB * ND;
+  constexpr int NMX = NC > ND ? NC : ND;
   for (int x = lane; x < N4; x += 32) {
-    double s0 = 0.0, s1 = 0.0;
+    int base, stride, cnt;
     size_t dst;
-    double* Kp = K;
     if (x < N1) {
       const int i = x / NC, k = x % NC;
-      for (int j = 0; j < NB; ++j)
-#pragma unroll
-        for (int l = 0; l < ND; ++l) {
-          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dbd[j * ND + l];
-          if (l & 1) s1 += t; else s0 += t;
-        }
-      dst = (size_t)(oa + i) * nbf + oc + k;
+      base = DL::PAC + i * NCD + k * ND; stride = 1; cnt = ND; dst = (size_t)(oa + i) * nbf + oc + k;
     } else if (x < N2) {
-      const int y = x - N1, i = y / ND, l = y % ND;
-      for (int j = 0; j < NB; ++j)
-#pragma unroll
-        for (int k = 0; k < NC; ++k) {
-          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dbc[j * NC + k];
-          if (k & 1) s1 += t; else s0 += t;
-        }
-      dst = (size_t)(oa + i) * nbf + od + l;
+      const int i = (x - N1) / ND, l = (x - N1) % ND;
+      base = DL::PAD + i * NCD + l; stride = ND; cnt = NC; dst = (size_t)(oa + i) * nbf + od + l;
     } else if (x < N3) {
-      const int y = x - N2, j = y / NC, k = y % NC;
-      for (int i = 0; i < NA; ++i)
-#pragma unroll
-        for (int l = 0; l < ND; ++l) {
-          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dad[i * ND + l];
-          if (l & 1) s1 += t; else s0 += t;
-        }
-      dst = (size_t)(ob + j) * nbf + oc + k;
+      const int j = (x - N2) / NC, k = (x - N2) % NC;
+      base = DL::PBC + j * NCD + k * ND; stride = 1; cnt = ND; dst = (size_t)(ob + j) * nbf + oc + k;
     } else {
-      const int y = x - N3, j = y / ND, l = y % ND;
-      for (int i = 0; i < NA; ++i)
-#pragma unroll
-        for (int k = 0; k < NC; ++k) {
-          const double t = V[(i * NB + j) * NCD + k * ND + l] * Dac[i * NC + k];
-          if (k & 1) s1 += t; else s0 += t;
-        }
-      dst = (size_t)(ob + j) * nbf + od + l;
+      const int j = (x - N3) / ND, l = (x - N3) % ND;
+      base = DL::PBD + j * NCD + l; stride = ND; cnt = NC; dst = (size_t)(ob + j) * nbf + od + l;
     }
-    atomicAdd(Kp + dst, deg * (s0 + s1));
+    double s = 0.0;
+#pragma unroll
+    for (int k = 0; k < NMX; ++k)
+      if (k < cnt) s += Ps[base + k * stride];
+    atomicAdd(K + dst, deg * s);
   }
   __syncwarp();
 }

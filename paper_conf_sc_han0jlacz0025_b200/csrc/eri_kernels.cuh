@@ -39,7 +39,7 @@ __host__ __device__ constexpr size_t cta_smem_bytes() {
 // occupancy cap (4 CTAs/SM, <= 128 registers) measured faster for the fd-bra classes and (fp|dd) only
 template <int X, int Y>
 constexpr int jk_minb() {
-  return (X == 8 || (X == 7 && Y == 5)) ? 4 : 1;
+  return in_list(kJkCap4, X * 100 + Y) ? 4 : 1;
 }
 
 // Persistent J/K kernel: each warp pulls tasks (bra pair, <= KT consecutive kets) from a global counter.
@@ -76,10 +76,10 @@ __device__ __forceinline__ void jk_body(const JKArgs& a) {
   const long long tg0 = a.task_begin + (long long)grab;
   if (tg0 >= a.task_end) break;
   const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
-  int U = find_bra(a.task_off, a.nbra, tg0);
+  int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;
-    const int P = U / a.ngroup;  // flat index = bra pair x ket primitive-count group
+    const int P = __ldg(a.ent_P + U);
     const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * a.KT;
     const int r1 = min(r0 + a.KT, __ldg(a.kend + U));
     const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
@@ -88,14 +88,18 @@ __device__ __forceinline__ void jk_body(const JKArgs& a) {
     for (int i = lane; i < C::NAB; i += 32) jab[i] = 0.0;
     __syncwarp();
     for (int R = r0; R < r1; ++R) {
-      if (QP * __ldg(a.ket.Q + R) < a.thresh) continue;
+      const double QQ = QP * __ldg(a.ket.Q + R);
+      if (QQ < a.thresh) continue;
       const int sc = __ldg(a.ket.shA + R), sd = __ldg(a.ket.shB + R);
+      if (!dw_keep(a, QQ, sa, sb, sc, sd)) continue;
+      const int oc = __ldg(a.ao + sc), od = __ldg(a.ao + sd);
+      d_prefetch<C>(jab + C::NAB, a.D, oa, ob, oc, od, a.nbf, lane);
       quartet_block<C>(a.bra, P, a.ket, R, Rbuf, V, htab, rtab, a.boys, lane);
       double deg = 1.0;
       if (sa == sb) deg *= 0.5;
       if (sc == sd) deg *= 0.5;
       if (a.same_bucket && P == R) deg *= 0.5;
-      digest<C>(V, deg, oa, ob, __ldg(a.ao + sc), __ldg(a.ao + sd), a.D, a.nbf, a.J, a.K, jab, jab + C::NAB, lane);
+      digest<C, false>(V, deg, oa, ob, oc, od, a.D, a.nbf, a.J, a.K, jab, jab + C::NAB, Rbuf, lane);
       __syncwarp();
     }
     for (int ab = lane; ab < C::NAB; ab += 32)

@@ -24,9 +24,11 @@ struct KfCfg {
   static constexpr int wpart(int nk) { return ((C::NHAB + (32 / nk) - 1) / (32 / nk)) * C::NCD; }
   static constexpr int regs(int nk) { return nH(C::L) + wpart(nk) + vfr(nk); }
   static constexpr int pick() {
-    return (vfr(16) <= 24 && regs(16) <= 128) ? 16
-                                              : ((vfr(8) <= 24 && regs(8) <= 128) ? 8
-                                                                                  : ((vfr(4) <= 24 && regs(4) <= 128) ? 4 : 0));
+    return (vfr(16) <= 24 && regs(16) <= 128)  ? 16
+           : (vfr(8) <= 24 && regs(8) <= 128)  ? 8
+           : (vfr(4) <= 24 && regs(4) <= 128)  ? 4
+           : (vfr(2) <= 24 && regs(2) <= 136)  ? 2
+                                               : 0;
   }
   static constexpr int NK = pick();                      // kets per warp task
   static constexpr int LPK = NK ? 32 / NK : 1;           // lanes per ket
@@ -36,21 +38,21 @@ struct KfCfg {
   static constexpr int WS = COLS + ((4 - COLS % 16) + 16) % 16;  // row stride = 4 (mod 16): conflict-free B loads
   static constexpr int ROWS = (C::MT * 8 > C::KS1 * 4) ? C::MT * 8 : C::KS1 * 4;
   static constexpr int WARP_DBL = ROWS * WS;
-  static constexpr size_t SMEM = sizeof(double) * 4 * WARP_DBL;
+  // per-ket D slots (D_cd | D_bd | D_bc | D_ad | D_ac, odd stride) + per-warp D_ab, filled by cp.async
+  static constexpr int OCD = 0, OBD = OCD + C::NCD, OBC = OBD + C::NB * C::ND, OAD = OBC + C::NB * C::NC,
+                       OAC = OAD + C::NA * C::ND, NDK = OAC + C::NA * C::NC, NDKS = NDK | 1;
+  static constexpr int WARP_D = (NK > 0 ? NK : 1) * NDKS + C::NAB;
+  static constexpr size_t SMEM = sizeof(double) * 4 * (WARP_DBL + WARP_D);
   static constexpr bool OK = NK > 0 && C::NHCD * C::NCD <= 140 && C::L <= 6;
   // 3 CTAs/SM (<= 168 registers, some spills) measured faster for these instantiations, else no cap
-  static constexpr int MINB = (X * 10 + Y == 41 || X * 10 + Y == 23 || X * 10 + Y == 71 || X * 10 + Y == 80 ||
-                               X * 10 + Y == 33 || X * 10 + Y == 90) ? 3 : 1;
+  static constexpr int MINB = in_list(kKfCap3, X * 100 + Y) ? 3 : 1;
 };
 
 template <int X, int Y>
 constexpr bool use_kf() {
   // measured per class on the valinomycin-sized workload (profiles/README.md): KF wins for light kets
   // with a heavier bra; pp kets (8-fold redundant R per ket) stay on the slot-batched kernel
-  constexpr int c = X * 100 + Y;
-  constexpr bool pick = c == 303 || c == 401 || c == 403 || c == 501 || c == 603 || c == 701 || c == 800 ||
-                        c == 801 || c == 900 || c == 700 || c == 500;
-  return KfCfg<X, Y>::OK && pick;
+  return KfCfg<X, Y>::OK && in_list(kKfPick, X * 100 + Y);
 }
 
 // Transposed execution of class (X|Y), X > Y: the task pair comes from bucket Y and the lanes take
@@ -58,9 +60,7 @@ constexpr bool use_kf() {
 // lighter side contracted per lane.  Used when the canonical ket has more functions than the bra.
 template <int X, int Y>
 constexpr bool use_kf_swap() {
-  constexpr int c = X * 100 + Y;
-  constexpr bool pick = c == 302;
-  if constexpr (X != Y) return KfCfg<Y, X>::OK && pick;
+  if constexpr (X != Y) return KfCfg<Y, X>::OK && in_list(kKfSwapPick, X * 100 + Y);
   return false;
 }
 
@@ -88,6 +88,8 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
   const int g = lane >> 2, t = lane & 3;
   const int kk = lane / LPK, hh = lane % LPK;
   double* Ws = kf_smem + (size_t)warp * K::WARP_DBL;
+  double* Dk = kf_smem + (size_t)4 * K::WARP_DBL + (size_t)warp * K::WARP_D + kk * K::NDKS;  // my ket's D slots
+  double* Dab_s = kf_smem + (size_t)4 * K::WARP_DBL + (size_t)warp * K::WARP_D + NK * K::NDKS;
   for (int i = lane; i < K::WARP_DBL; i += 32) Ws[i] = 0.0;  // padding rows/cols stay zero forever
   __syncwarp();
   for (;;) {
@@ -97,19 +99,39 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
   const long long tg0 = a.task_begin + (long long)grab;
   if (tg0 >= a.task_end) break;
   const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
-  int U = find_bra(a.task_off, a.nbra, tg0);
+  int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;
-    const int P = U / a.ngroup;  // flat index = bra pair x ket primitive-count group
+    const int P = __ldg(a.ent_P + U);
     const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * NK;
     const int r1 = min(r0 + NK, __ldg(a.kend + U));
     const int R = r0 + kk;
     const double QP = __ldg(a.bra.Q + P);
-    const bool active = R < r1 && QP * __ldg(a.ket.Q + min(R, r1 - 1)) >= a.thresh;
+    const double QQ = QP * __ldg(a.ket.Q + min(R, r1 - 1));
     const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
+    const bool active = R < r1 && QQ >= a.thresh &&
+                        dw_keep(a, QQ, sa, sb, __ldg(a.ket.shA + min(R, r1 - 1)), __ldg(a.ket.shB + min(R, r1 - 1)));
     const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
     const int b0 = __ldg(a.bra.poff + P), b1 = __ldg(a.bra.poff + P + 1);
     const int k0 = active ? __ldg(a.ket.poff + R) : 0, k1 = active ? __ldg(a.ket.poff + R + 1) : 0;
+    const int sc = active ? __ldg(a.ket.shA + R) : 0, sd = active ? __ldg(a.ket.shB + R) : 0;
+    const int oc = active ? __ldg(a.ao + sc) : 0, od = active ? __ldg(a.ao + sd) : 0;
+    {
+      // D sub-blocks of this task's quartets: asynchronous copies, waited for before the digestion
+      const size_t nb = (size_t)a.nbf;
+      for (int x = lane; x < NAB; x += 32) cp_async8(Dab_s + x, a.D + (oa + x / NB) * nb + ob + x % NB);
+      if (active)
+        for (int x = hh; x < K::NDK; x += LPK) {
+          int r, c;
+          if (x < K::OBD) { r = oc + x / ND; c = od + x % ND; }
+          else if (x < K::OBC) { r = ob + (x - K::OBD) / ND; c = od + (x - K::OBD) % ND; }
+          else if (x < K::OAD) { r = ob + (x - K::OBC) / NC; c = oc + (x - K::OBC) % NC; }
+          else if (x < K::OAC) { r = oa + (x - K::OAD) / ND; c = od + (x - K::OAD) % ND; }
+          else { r = oa + (x - K::OAC) / NC; c = oc + (x - K::OAC) % NC; }
+          cp_async8(Dk + x, a.D + (size_t)r * nb + c);
+        }
+      cp_async_commit();
+    }
     double vf[MT][NTV][2];
 #pragma unroll
     for (int m = 0; m < MT; ++m)
@@ -190,25 +212,22 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
         }
     __syncwarp();
     // ---- digestion (a9) ----
-    const int sc = active ? __ldg(a.ket.shA + R) : 0, sd = active ? __ldg(a.ket.shB + R) : 0;
     double deg = 1.0;
     if (sa == sb) deg *= 0.5;
     if (sc == sd) deg *= 0.5;
     if (a.same_bucket && P == R) deg *= 0.5;
     if (!active) deg = 0.0;
-    const int oc = active ? __ldg(a.ao + sc) : 0, od = active ? __ldg(a.ao + sd) : 0;
-    const double* __restrict__ Dm = a.D;
     const size_t nb = (size_t)a.nbf;
     const double* Vk = Ws + kk * NCD;  // V[ab][cd] of my ket = Vk[ab * WS + cd]
+    cp_async_wait_all();
+    __syncwarp();
     // J_ab: lanes with the same hh share ab; reduce over the kets
     for (int i0 = 0; i0 < NAB; i0 += LPK) {
       const int ab = i0 + hh;
       double s = 0.0;
       if (active && ab < NAB) {
 #pragma unroll
-        for (int k = 0; k < NC; ++k)
-#pragma unroll
-          for (int l = 0; l < ND; ++l) s = fma(Vk[ab * WS + k * ND + l], __ldg(Dm + (oc + k) * nb + od + l), s);
+        for (int x = 0; x < NCD; ++x) s = fma(Vk[ab * WS + x], Dk[K::OCD + x], s);
       }
       s *= deg;
 #pragma unroll
@@ -219,8 +238,8 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
       // J_cd
       for (int cd = hh; cd < NCD; cd += LPK) {
         double s = 0.0;
-        for (int i = 0; i < NA; ++i)
-          for (int j = 0; j < NB; ++j) s = fma(Vk[(i * NB + j) * WS + cd], __ldg(Dm + (oa + i) * nb + ob + j), s);
+#pragma unroll
+        for (int ij = 0; ij < NAB; ++ij) s = fma(Vk[ij * WS + cd], Dab_s[ij], s);
         atomicAdd(a.J + (oc + cd / ND) * nb + od + cd % ND, 2.0 * deg * s);
       }
       // K_ac (NA*NC) | K_ad (NA*ND) | K_bc (NB*NC) | K_bd (NB*ND), flattened over the lanes of the ket
@@ -230,22 +249,22 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
         if (x < N1) {
           const int i = x / NC, k = x % NC;
           for (int j = 0; j < NB; ++j)
-            for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (ob + j) * nb + od + l), s);
+            for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OBD + j * ND + l], s);
           atomicAdd(a.K + (oa + i) * nb + oc + k, deg * s);
         } else if (x < N2) {
           const int y = x - N1, i = y / ND, l = y % ND;
           for (int j = 0; j < NB; ++j)
-            for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (ob + j) * nb + oc + k), s);
+            for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OBC + j * NC + k], s);
           atomicAdd(a.K + (oa + i) * nb + od + l, deg * s);
         } else if (x < N3) {
           const int y = x - N2, j = y / NC, k = y % NC;
           for (int i = 0; i < NA; ++i)
-            for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (oa + i) * nb + od + l), s);
+            for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OAD + i * ND + l], s);
           atomicAdd(a.K + (ob + j) * nb + oc + k, deg * s);
         } else {
           const int y = x - N3, j = y / ND, l = y % ND;
           for (int i = 0; i < NA; ++i)
-            for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], __ldg(Dm + (oa + i) * nb + oc + k), s);
+            for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OAC + i * NC + k], s);
           atomicAdd(a.K + (ob + j) * nb + od + l, deg * s);
         }
       }

@@ -37,7 +37,8 @@ struct SlabCfg {
   static constexpr int RCAP = 16;                 // R rows per warp (combos per R phase)
   static constexpr int RSTRIDE = C::NH | 1;       // odd row stride (doubles)
   // warp SMEM (doubles): R rows, V for NS kets, J_ab partial
-  static constexpr int W_R = RCAP * RSTRIDE;
+  // R rows; doubles as the digestion partial-sum scratch
+  static constexpr int W_R = (RCAP * RSTRIDE > 2 * (C::NA + C::NB) * C::NCD) ? RCAP * RSTRIDE : 2 * (C::NA + C::NB) * C::NCD;
   static constexpr int W_V = NS * C::NAB * C::NCD;
   static constexpr int WARP_DBL = W_R + W_V + C::NAB + 2 + C::W_D;
   // CTA table: B-fragment offsets [KS1][NT1B][32] (slot << 10 | hermite index, -1 = zero)
@@ -49,7 +50,7 @@ template <int X, int Y>
 constexpr bool use_slab() {
   // measured per class (profiles/README.md): only (pp|pp) and (dp|pp) -- bras with up to 16 primitive
   // pairs and pp kets -- still beat the warp-per-quartet kernel with its once-per-quartet R rows
-  return !use_tpq(X, Y) && SlabCfg<X, Y>::OK && ((X == 2 && Y == 2) || (X == 4 && Y == 2));
+  return !use_tpq(X, Y) && SlabCfg<X, Y>::OK && in_list(kSlabPick, X * 100 + Y);
 }
 
 template <int X, int Y>
@@ -89,10 +90,10 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
   const long long tg0 = a.task_begin + (long long)grab;
   if (tg0 >= a.task_end) break;
   const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
-  int U = find_bra(a.task_off, a.nbra, tg0);
+  int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;
-    const int P = U / a.ngroup;  // flat index = bra pair x ket primitive-count group
+    const int P = __ldg(a.ent_P + U);
     const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * a.KT;
     const int r1 = min(r0 + a.KT, __ldg(a.kend + U));
     const double QP = __ldg(a.bra.Q + P);
@@ -112,7 +113,8 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
       int ns = 0, nvk = 0;
       const bool cont = kl != __ldg(a.ket.poff + r);  // batch starts inside a ket (V row carries over)
       while (ns < nsl && r < r1) {
-        if (QP * __ldg(a.ket.Q + r) < a.thresh) {  // (prefix already respects thresh; kept for safety)
+        const double QQ = QP * __ldg(a.ket.Q + r);
+        if (QQ < a.thresh || !dw_keep(a, QQ, sa, sb, __ldg(a.ket.shA + r), __ldg(a.ket.shB + r))) {
           ++r;
           if (r < r1) kl = __ldg(a.ket.poff + r);
           continue;
@@ -244,7 +246,7 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
         if (sc == sd) deg *= 0.5;
         if (a.same_bucket && P == R) deg *= 0.5;
         digest<C>(Vs + (size_t)v * NAB * NCD, deg, oa, ob, __ldg(a.ao + sc), __ldg(a.ao + sd), a.D, a.nbf, a.J, a.K,
-                  jab, jab + NAB + 2, lane);
+                  jab, jab + NAB + 2, Rs, lane);
         __syncwarp();
       }
     }

@@ -126,18 +126,32 @@ constexpr bool tpq_wacc() {
 
 constexpr int TASK_GRAB = 4;  // tasks taken per counter increment (one bra search per grab)
 
-__device__ __forceinline__ int find_bra(const long long* __restrict__ task_off, int nbra, long long task) {
-  int lo = 0, hi = nbra - 1;
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if (__ldg(task_off + mid) <= task) lo = mid; else hi = mid - 1;
-  }
-  return lo;
+// density-weighted screening of quartet (sa sb|sc sd) with Schwarz product qq (reading R17)
+__device__ __forceinline__ bool dw_keep(const JKArgs& a, double qq, int sa, int sb, int sc, int sd) {
+  if (a.dsh == nullptr) return true;
+  const float* __restrict__ t = a.dsh;
+  const size_t n = (size_t)a.nshell;
+  const float m = fmaxf(fmaxf(__ldg(t + sa * n + sb), __ldg(t + sc * n + sd)),
+                        fmaxf(fmaxf(__ldg(t + sa * n + sc), __ldg(t + sa * n + sd)),
+                              fmaxf(__ldg(t + sb * n + sc), __ldg(t + sb * n + sd))));
+  return qq * (double)m * (1.0 + 1e-6) >= a.dw_thresh;  // (float rounding of the block maxima)
+}
+
+// entry (non-empty bra pair x ket K-group) holding task `task`: sampled start + short forward scan
+__device__ __forceinline__ int find_entry(const JKArgs& a, long long task) {
+  int U = __ldg(a.usamp + (task >> TASK_SAMPLE_SHIFT));
+  while (__ldg(a.task_off + U + 1) <= task) ++U;
+  return U;
 }
 
 // Persistent lane-per-ket kernel (JKArgs.KT must be 32).
+#ifdef MAKO_TPQ_MINB
+#define MAKO_TPQ_BOUNDS __launch_bounds__(128, MAKO_TPQ_MINB)
+#else
+#define MAKO_TPQ_BOUNDS __launch_bounds__(128)
+#endif
 template <int X, int Y>
-__global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
+__global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
   using C = ClsXY<X, Y>;
   constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
   constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND;
@@ -150,16 +164,18 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
   const long long tg0 = a.task_begin + (long long)grab;
   if (tg0 >= a.task_end) break;
   const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
-  int U = find_bra(a.task_off, a.nbra, tg0);
+  int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;
-    const int P = U / a.ngroup;  // flat index = bra pair x ket primitive-count group
+    const int P = __ldg(a.ent_P + U);
     const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * 32;
     const int r1 = min(r0 + 32, __ldg(a.kend + U));
     const int R = r0 + lane;
     const double QP = __ldg(a.bra.Q + P);
-    const bool active = R < r1 && QP * __ldg(a.ket.Q + min(R, r1 - 1)) >= a.thresh;
+    const double QQ = QP * __ldg(a.ket.Q + min(R, r1 - 1));
     const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
+    const bool active = R < r1 && QQ >= a.thresh &&
+                        dw_keep(a, QQ, sa, sb, __ldg(a.ket.shA + min(R, r1 - 1)), __ldg(a.ket.shB + min(R, r1 - 1)));
     const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
     const int b0 = __ldg(a.bra.poff + P), b1 = __ldg(a.bra.poff + P + 1);
     double V[NAB][NCD];
@@ -171,6 +187,8 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
     if (active) {
       sc = __ldg(a.ket.shA + R);
       sd = __ldg(a.ket.shB + R);
+    }
+    if (active) {
       const int k0 = __ldg(a.ket.poff + R), k1 = __ldg(a.ket.poff + R + 1);
       if constexpr (WACC) {
         // bra primitive outer: W[p][cd] = sum_kl sum_q R_{p+q} E~_cd[q][cd], then V += E~_ab W
@@ -252,18 +270,16 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
     if (sc == sd) deg *= 0.5;
     if (a.same_bucket && P == R) deg *= 0.5;
     if (!active) deg = 0.0;
-    const double* __restrict__ Dm = a.D;
     const size_t n = (size_t)a.nbf;
     const int oc = active ? __ldg(a.ao + sc) : 0, od = active ? __ldg(a.ao + sd) : 0;
+    const double* __restrict__ Dm = a.D;
     // J_ab: per-lane deg-weighted partial, warp reduction over the 32 kets, one atomic per element
 #pragma unroll
     for (int i = 0; i < NAB; ++i) {
       double s = 0.0;
       if (active) {
 #pragma unroll
-        for (int k = 0; k < NC; ++k)
-#pragma unroll
-          for (int l = 0; l < ND; ++l) s = fma(V[i][k * ND + l], __ldg(Dm + (oc + k) * n + od + l), s);
+        for (int kl = 0; kl < NCD; ++kl) s = fma(V[i][kl], __ldg(Dm + (oc + kl / ND) * n + od + kl % ND), s);
       }
       s *= deg;
 #pragma unroll
@@ -278,9 +294,7 @@ __global__ void __launch_bounds__(128) tpq_jk_kernel(JKArgs a) {
       for (int l = 0; l < ND; ++l) {
         double s = 0.0;
 #pragma unroll
-        for (int i = 0; i < NA; ++i)
-#pragma unroll
-          for (int j = 0; j < NB; ++j) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (oa + i) * n + ob + j), s);
+        for (int ij = 0; ij < NAB; ++ij) s = fma(V[ij][k * ND + l], __ldg(Dm + (oa + ij / NB) * n + ob + ij % NB), s);
         atomicAdd(a.J + (oc + k) * n + od + l, 2.0 * deg * s);
       }
     // K_ac += v D_bd ; K_ad += v D_bc ; K_bc += v D_ad ; K_bd += v D_ac

@@ -78,6 +78,16 @@ static int prefix_count(const std::vector<double>& QY, int lo0, int hi0, double 
 
 static mako_status ensure_plan(mako_pairs P, double thresh) {
   if (P->plan.thresh == thresh && !P->plan.cls.empty()) return MAKO_OK;
+  for (auto& sp : P->plan_cache)
+    if (sp.thresh == thresh && !sp.cls.empty()) {
+      std::swap(P->plan, sp);
+      return MAKO_OK;
+    }
+  if (!P->plan.cls.empty()) {
+    P->plan_cache.push_back(std::move(P->plan));
+    if (P->plan_cache.size() > 6) P->plan_cache.erase(P->plan_cache.begin());
+  }
+  P->plan = Plan();
   Plan& pl = P->plan;
   pl.cls.clear();
   pl.cls.resize(NBUCKET * (NBUCKET + 1) / 2);
@@ -94,24 +104,33 @@ static mako_status ensure_plan(mako_pairs P, double thresh) {
       const PairBucket& bx = P->set.b[c.TB];
       const PairBucket& by = P->set.b[c.LB];
       const int nbra = bx.n(), G = NKGROUP;
-      c.kbeg.assign((size_t)nbra * G, 0);
-      c.kend.assign((size_t)nbra * G, 0);
-      c.task_off.assign((size_t)nbra * G + 1, 0);
+      c.ent_P.clear();
+      c.kbeg.clear();
+      c.kend.clear();
+      c.task_off.assign(1, 0);
       for (int p = 0; p < nbra; ++p)
         for (int g = 0; g < G; ++g) {
-          const size_t u = (size_t)p * G + g;
           const int s0 = by.seg.empty() ? 0 : by.seg[g], s1 = by.seg.empty() ? (g == 0 ? by.n() : 0) : by.seg[g + 1];
           int nk = s1 > s0 ? prefix_count(by.Q, s0, s1, bx.Q[p], thresh) : 0;
           if (X == Y) nk = std::min(nk, std::max(0, p - s0 + 1));  // canonical: ket position <= bra position
-          c.kbeg[u] = s0;
-          c.kend[u] = s0 + nk;
+          if (nk <= 0) continue;
+          c.ent_P.push_back(p);
+          c.kbeg.push_back(s0);
+          c.kend.push_back(s0 + nk);
           c.nquartet += nk;
-          c.task_off[u + 1] = c.task_off[u] + (nk + c.KT - 1) / c.KT;
+          c.task_off.push_back(c.task_off.back() + (nk + c.KT - 1) / c.KT);
         }
-      c.ntask = c.task_off[(size_t)nbra * G];
+      c.ntask = c.task_off.back();
+      c.usamp.assign((size_t)(c.ntask >> TASK_SAMPLE_SHIFT) + 1, 0);
+      for (size_t u = 0, k = 0; k < c.usamp.size(); ++k) {
+        const long long t = (long long)k << TASK_SAMPLE_SHIFT;
+        while (u + 1 < c.ent_P.size() && c.task_off[u + 1] <= t) ++u;
+        c.usamp[k] = (int)u;
+      }
       mako_status st;
       if (c.ntask > 0 && ((st = upload(c.d_kbeg, c.kbeg)) || (st = upload(c.d_kend, c.kend)) ||
-                          (st = upload(c.d_task_off, c.task_off))))
+                          (st = upload(c.d_task_off, c.task_off)) || (st = upload(c.d_ent_P, c.ent_P)) ||
+                          (st = upload(c.d_usamp, c.usamp))))
         return st;
     }
   pl.thresh = thresh;
@@ -129,6 +148,25 @@ __global__ void symmetrize_kernel(double* __restrict__ J, double* __restrict__ K
     J[a] = sj; J[b] = sj;
     K[a] = sk; K[b] = sk;
   }
+}
+
+// density screening: dsh[sa][sb] = max |D| over the (sa, sb) block (rounded up to float); dmax = max |D|
+__global__ void dsh_kernel(const double* __restrict__ D, int nbf, int nshell, const int* __restrict__ ao,
+                           const int* __restrict__ l, float* __restrict__ dsh, unsigned long long* __restrict__ dmax) {
+  const long long n2 = (long long)nshell * nshell;
+  double gm = 0.0;
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < n2; x += (long long)gridDim.x * blockDim.x) {
+    const int sa = (int)(x / nshell), sb = (int)(x % nshell);
+    const int oa = ao[sa], ob = ao[sb], na = 2 * l[sa] + 1, nb = 2 * l[sb] + 1;
+    double m = 0.0;
+    for (int i = 0; i < na; ++i)
+      for (int j = 0; j < nb; ++j) m = fmax(m, fabs(D[(size_t)(oa + i) * nbf + ob + j]));
+    dsh[x] = __double2float_ru(m);
+    gm = fmax(gm, m);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) gm = fmax(gm, __shfl_xor_sync(0xffffffffu, gm, o));
+  if ((threadIdx.x & 31) == 0) atomicMax(dmax, (unsigned long long)__double_as_longlong(gm));  // gm >= 0
 }
 
 __global__ void boys_kernel(int n, const double* __restrict__ T, double* __restrict__ out, const double* __restrict__ tab,
@@ -209,11 +247,10 @@ static mako_status class_flops(mako_pairs p, double thresh, int shard, int nshar
     const double hab = nH(la + lb), hcd = nH(lc + ld);
     const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
     // surviving kets of each (bra, K-group) entry restricted to this shard's tasks
-    const int G = NKGROUP;
     for (size_t u = 0; u < c.kbeg.size(); ++u) {
       const long long a0 = c.task_off[u], a1 = c.task_off[u + 1];
       if (a1 <= t0 || a0 >= t1) continue;
-      const int Pb = (int)(u / G);
+      const int Pb = c.ent_P[u];
       const long long KAB = bx.poff[Pb + 1] - bx.poff[Pb];
       const int r0 = c.kbeg[u] + (int)(std::max(a0, t0) - a0) * KT;
       const int r1 = std::min(c.kbeg[u] + (int)(std::min(a1, t1) - a0) * KT, c.kend[u]);
@@ -345,8 +382,8 @@ extern "C" mako_status mako_build_jk_launches(mako_pairs p, double thresh, int s
   return MAKO_OK;
 }
 
-extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thresh, double* J, double* K, int shard,
-                                     int nshards, void* cuda_stream) {
+static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, unsigned flags, double* J, double* K,
+                                 int shard, int nshards, void* cuda_stream) {
   try {
     mako_status st;
     if ((st = check_pairs(p))) return st;
@@ -354,11 +391,31 @@ extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thres
     if (D == J || D == K || J == K) return fail(MAKO_ERR_INVALID, "D, J, K must not alias");
     if (!(thresh >= 0) || !std::isfinite(thresh)) return fail(MAKO_ERR_INVALID, "thresh must be finite and >= 0");
     if (nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "shard out of range");
-    thresh = std::max(thresh, p->tau);
-    if ((st = ensure_plan(p, thresh))) return st;
+    if (flags & ~(unsigned)MAKO_JK_DENSITY_SCREEN) return fail(MAKO_ERR_INVALID, "unknown flags");
     const mako_basis_s* B = p->basis;
     const int n = B->nbf;
     cudaStream_t s = (cudaStream_t)cuda_stream;
+    const bool dw = (flags & MAKO_JK_DENSITY_SCREEN) != 0;
+    const double dw_thresh = std::max(thresh, p->tau);
+    if (dw) {
+      // shell-block maxima of |D| and the global max; the task plan is the Schwarz prefix at
+      // thresh / max|D| rounded down to a power of ten (a superset of the density-screened quartets,
+      // few distinct plans over an SCF run), each quartet is then tested in the kernels
+      const int ns = B->nshell;
+      if (!p->d_dsh.p && (st = p->d_dsh.alloc(sizeof(float) * (size_t)ns * ns))) return st;
+      if (!p->d_dmax.p && (st = p->d_dmax.alloc(sizeof(double)))) return st;
+      if ((st = cuda_check(cudaMemsetAsync(p->d_dmax.p, 0, sizeof(double), s), "memset dmax"))) return st;
+      dsh_kernel<<<592, 256, 0, s>>>(D, n, ns, B->d_ao.as<int>(), B->d_l.as<int>(), p->d_dsh.as<float>(),
+                                     p->d_dmax.as<unsigned long long>());
+      double dmax = 0.0;
+      if ((st = cuda_check(cudaMemcpyAsync(&dmax, p->d_dmax.p, sizeof(double), cudaMemcpyDeviceToHost, s), "dmax")) ||
+          (st = cuda_check(cudaStreamSynchronize(s), "dmax sync")))
+        return st;
+      if (!std::isfinite(dmax)) return fail(MAKO_ERR_INVALID, "D is not finite");
+      thresh = dmax > 0 ? std::pow(10.0, std::floor(std::log10(dw_thresh / dmax))) : 1e300;
+    }
+    thresh = std::max(thresh, p->tau);
+    if ((st = ensure_plan(p, thresh))) return st;
     if ((st = cuda_check(cudaMemsetAsync(J, 0, sizeof(double) * n * n, s), "memset J")) ||
         (st = cuda_check(cudaMemsetAsync(K, 0, sizeof(double) * n * n, s), "memset K")) ||
         (st = cuda_check(cudaMemsetAsync(p->d_counters.p, 0, sizeof(unsigned long long) * 64, s), "memset ctr")))
@@ -394,8 +451,9 @@ extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thres
       a.task_off = c.d_task_off.as<long long>();
       a.kbeg = c.d_kbeg.as<int>();
       a.kend = c.d_kend.as<int>();
-      a.nbra = (int)c.kbeg.size();
-      a.ngroup = NKGROUP;
+      a.ent_P = c.d_ent_P.as<int>();
+      a.usamp = c.d_usamp.as<int>();
+      a.nent = (int)c.kbeg.size();
       a.KT = c.KT;
       a.counter = p->d_counters.as<unsigned long long>() + class_index(c.X, c.Y);
       a.D = D;
@@ -404,6 +462,9 @@ extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thres
       a.nbf = n;
       a.ao = B->d_ao.as<int>();
       a.thresh = thresh;
+      a.dsh = dw ? p->d_dsh.as<float>() : nullptr;
+      a.nshell = B->nshell;
+      a.dw_thresh = dw_thresh;
       a.boys = B->d_boys.as<double>();
       a.grid_div = 1;
       cudaEvent_t e0 = nullptr, e1 = nullptr;
@@ -428,6 +489,16 @@ extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thres
   } catch (const std::exception& e) {
     return fail(MAKO_ERR_OOM, e.what());
   }
+}
+
+extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thresh, double* J, double* K, int shard,
+                                     int nshards, void* cuda_stream) {
+  return build_jk_impl(p, D, thresh, 0u, J, K, shard, nshards, cuda_stream);
+}
+
+extern "C" mako_status mako_build_jk_ex(mako_pairs p, const double* D, double thresh, unsigned flags, double* J,
+                                        double* K, int shard, int nshards, void* cuda_stream) {
+  return build_jk_impl(p, D, thresh, flags, J, K, shard, nshards, cuda_stream);
 }
 
 extern "C" mako_status mako_eri_batch(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,

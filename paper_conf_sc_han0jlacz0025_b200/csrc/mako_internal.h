@@ -75,6 +75,39 @@ MK_HD constexpr int kgroup(int K) {
                 : (K <= 6 ? 4 : (K <= 9 ? 5 : (K <= 12 ? 6 : (K <= 16 ? 7 : (K <= 24 ? 8 : (K <= 36 ? 9 : 10))))));
 }
 
+// Per-class kernel-family choices, measured on the bench workload (profiles/README.md).  Codes are
+// X * 100 + Y.  Overridable with -D for experiment builds (build.py --variant).
+#ifndef MAKO_KF_PICK
+#define MAKO_KF_PICK 303, 401, 403, 501, 603, 701, 800, 801, 900, 700, 500
+#endif
+#ifndef MAKO_KFSWAP_PICK
+#define MAKO_KFSWAP_PICK 302
+#endif
+#ifndef MAKO_SLAB_PICK
+#define MAKO_SLAB_PICK 202, 402
+#endif
+#ifndef MAKO_JK_CAP4
+#define MAKO_JK_CAP4 800, 801, 802, 803, 804, 805, 806, 807, 808, 705
+#endif
+#ifndef MAKO_KF_CAP3
+#define MAKO_KF_CAP3 401, 203, 701, 800, 303, 900
+#endif
+constexpr int kKfPick[] = {MAKO_KF_PICK};
+constexpr int kKfSwapPick[] = {MAKO_KFSWAP_PICK};
+constexpr int kSlabPick[] = {MAKO_SLAB_PICK};
+constexpr int kJkCap4[] = {MAKO_JK_CAP4};
+constexpr int kKfCap3[] = {MAKO_KF_CAP3};
+template <int N>
+MK_HD constexpr bool in_list(const int (&a)[N], int v) {
+  for (int i = 0; i < N; ++i)
+    if (a[i] == v) return true;
+  return false;
+}
+
+// task -> entry lookup: every TASK_SAMPLE-th task's entry is stored, the rest is a short forward scan
+constexpr int TASK_SAMPLE_SHIFT = 4;
+constexpr int TASK_SAMPLE = 1 << TASK_SAMPLE_SHIFT;
+
 // primitive-pair screening (reading R7)
 constexpr double PRIM_PAIR_EPS = 1e-18;
 
@@ -98,11 +131,12 @@ struct JKArgs {
   PairView bra, ket;
   int same_bucket;
   long long task_begin, task_end;   // shard range of this class's task index space
-  const long long* task_off;        // [nbra+1] task prefix per flat (bra pair, ket K-group) entry
-  const int* kbeg;                  // [nbra] first ket of the entry (start of its K-group segment)
-  const int* kend;                  // [nbra] one past the last surviving ket (Q-sorted prefix of the segment)
-  int nbra;                         // flat entries = bra pairs x ngroup
-  int ngroup;                       // ket primitive-count groups per bucket
+  const long long* task_off;        // [nent+1] task prefix per non-empty (bra pair, ket K-group) entry
+  const int* ent_P;                 // [nent] bra pair of the entry
+  const int* kbeg;                  // [nent] first ket of the entry (start of its K-group segment)
+  const int* kend;                  // [nent] one past the last surviving ket (Q-sorted prefix of the segment)
+  const int* usamp;                 // [ntask / TASK_SAMPLE + 1] entry holding task k * TASK_SAMPLE
+  int nent;
   int KT;                           // kets per task
   unsigned long long* counter;      // dynamic task counter (zeroed before launch)
   const double* D;
@@ -111,6 +145,11 @@ struct JKArgs {
   int nbf;
   const int* ao;                    // [nshell] AO offsets
   double thresh;
+  // density-weighted screening (flag MAKO_JK_DENSITY_SCREEN; null = off): keep a quartet iff
+  // Q_ab Q_cd max(|D| over its six shell blocks) >= dw_thresh; dsh[sa * nshell + sb] = max |D| of block
+  const float* dsh;
+  int nshell;
+  double dw_thresh;
   const double* boys;               // Boys table
   int grid_div;                     // host side: grid = resident capacity / grid_div (concurrent classes)
 };

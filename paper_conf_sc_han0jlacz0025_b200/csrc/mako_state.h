@@ -61,9 +61,11 @@ struct ClassPlan {
   int TB = 0, LB = 0;              // task bucket, lane bucket
   long long ntask = 0;             // tasks of the whole class (all shards)
   long long nquartet = 0;
-  std::vector<int> kbeg, kend;     // [nbra * NKGROUP]
-  std::vector<long long> task_off; // [nbra * NKGROUP + 1]
-  DevBuf d_kbeg, d_kend, d_task_off;
+  // non-empty (bra pair, ket K-group) entries, in (bra Q desc, group) order
+  std::vector<int> ent_P, kbeg, kend;  // [nent] bra pair, first / one-past-last surviving ket
+  std::vector<long long> task_off;     // [nent + 1] task prefix
+  std::vector<int> usamp;              // [ntask / TASK_SAMPLE + 1] entry holding task k * TASK_SAMPLE
+  DevBuf d_ent_P, d_kbeg, d_kend, d_task_off, d_usamp;
 };
 
 struct Plan {
@@ -91,8 +93,11 @@ struct mako_pairs_s {
   mako_basis basis = nullptr;   // not owned; must outlive the pairs
   double tau = 0.0;
   mako::PairSet set;
-  mako::Plan plan;
+  mako::Plan plan;                       // current plan
+  std::vector<mako::Plan> plan_cache;    // recently used plans of other thresholds (density screening)
   mako::DevBuf d_counters;      // [55] task counters
+  mako::DevBuf d_dsh;           // [nshell * nshell] float: max |D| per shell block (density screening)
+  mako::DevBuf d_dmax;          // [1] double: max |D| (density screening)
   // profiling (mako_profile_enable / read)
   bool prof = false;
   // concurrent class launches: internal streams forked from / joined to the caller's stream
