@@ -141,6 +141,8 @@ CONFIGS = {
     "h2o-sto3g": (h2o_baseline, "sto-3g"),
     "benzene-def2svp": (benzene, "def2-svp"),
     "gly10-ccpvtz": (lambda: glycine_oligomer(10), "cc-pvtz"),
+    # not a BASELINE config: the SCF-timing case of the incremental builder
+    "gly10-def2svp": (lambda: glycine_oligomer(10), "def2-svp"),
     "valinomycin-def2tzvp": (lambda: random_packed(VALINOMYCIN, name="valinomycin-sized"), "def2-tzvp"),
     "ubiquitin-def2tzvp": (lambda: random_packed(UBIQUITIN, name="ubiquitin-sized"), "def2-tzvp"),
 }

@@ -535,8 +535,25 @@ static void digest(const basis_t* B, int a, int b, int c, int d, const double* b
    (an oracle-side sample; the GPU library's own shard partition is not replicated here).
    Qin: optional precomputed Schwarz table (orc_schwarz), NULL to compute it here.
    J, K: [nbf][nbf] outputs (overwritten), final symmetrised values. */
+static int jk_impl(BASIS_ARGS, const double* Dm, double tau, double tau_dw, int shard, int nshards,
+                   const double* Qin, double* Jout, double* Kout);
+
 int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, const double* Qin, double* Jout,
            double* Kout) {
+  return jk_impl(nshell, l, nprim, xyz, exps, coefs, pure, Dm, tau, -1.0, shard, nshards, Qin, Jout, Kout);
+}
+
+/* Density-weighted screening ("density-weighted Schwarz"; reading R17):
+   as orc_jk, and a quartet is kept only if also Q_ab Q_cd Dmax >= tau_dw, where Dmax is the largest
+   max|D_mn| over the six shell blocks (ab)(cd)(ac)(ad)(bc)(bd) the quartet is contracted with. */
+int orc_jk_dw(BASIS_ARGS, const double* Dm, double tau, double tau_dw, const double* Qin, double* Jout,
+              double* Kout) {
+  if (!(tau_dw >= 0)) return 1;
+  return jk_impl(nshell, l, nprim, xyz, exps, coefs, pure, Dm, tau, tau_dw, 0, 1, Qin, Jout, Kout);
+}
+
+static int jk_impl(BASIS_ARGS, const double* Dm, double tau, double tau_dw, int shard, int nshards,
+                   const double* Qin, double* Jout, double* Kout) {
   BASIS_INIT(B);
   if (nshards < 1 || shard < 0 || shard >= nshards || tau < 0) { basis_free(&B); return 1; }
   int N = B.nbf;
@@ -554,6 +571,19 @@ int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, con
     for (int b = 0; b <= a; ++b, ++k) { pa[k] = a; pb[k] = b; }
   memset(Jout, 0, sizeof(double) * (size_t)N * N);
   memset(Kout, 0, sizeof(double) * (size_t)N * N);
+  /* shell-block maxima of |D| (density-weighted screening only) */
+  double* Dsh = (double*)calloc((size_t)nshell * nshell, sizeof(double));
+  if (tau_dw >= 0)
+    for (int x = 0; x < nshell; ++x)
+      for (int y = 0; y < nshell; ++y) {
+        double m = 0.0;
+        for (int i = 0; i < B.aoff[x + 1] - B.aoff[x]; ++i)
+          for (int j = 0; j < B.aoff[y + 1] - B.aoff[y]; ++j) {
+            double v = fabs(Dm[(size_t)(B.aoff[x] + i) * N + B.aoff[y] + j]);
+            if (v > m) m = v;
+          }
+        Dsh[x * nshell + y] = m;
+      }
 #pragma omp parallel
   {
     double* Jl = (double*)calloc((size_t)N * N, sizeof(double));
@@ -565,7 +595,15 @@ int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, con
       int a = pa[P], b = pb[P];
       for (int R = 0; R <= P; ++R) {
         int c = pa[R], d = pb[R];
-        if (Q[a * nshell + b] * Q[c * nshell + d] < tau) continue;
+        double qq = Q[a * nshell + b] * Q[c * nshell + d];
+        if (qq < tau) continue;
+        if (tau_dw >= 0) {
+          double m = Dsh[a * nshell + b];
+          double t[5] = {Dsh[c * nshell + d], Dsh[a * nshell + c], Dsh[a * nshell + d], Dsh[b * nshell + c],
+                         Dsh[b * nshell + d]};
+          for (int z = 0; z < 5; ++z) if (t[z] > m) m = t[z];
+          if (qq * m < tau_dw) continue;
+        }
         eri_block(&B, a, b, c, d, blk);
         double deg = 1.0;
         if (a == b) deg *= 0.5;
@@ -588,7 +626,7 @@ int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, con
       s = Kout[(size_t)i * N + j] + Kout[(size_t)j * N + i];
       Kout[(size_t)i * N + j] = Kout[(size_t)j * N + i] = s;
     }
-  free(Q); free(pa); free(pb);
+  free(Q); free(pa); free(pb); free(Dsh);
   basis_free(&B);
   return 0;
 }

@@ -109,6 +109,21 @@ def jk(sh, D, tau=0.0, shard=0, nshards=1, pure=True, Q=None):
     return J, K
 
 
+def jk_dw(sh, D, tau, tau_dw, pure=True, Q=None):
+    """J/K with the Schwarz rule at tau plus density-weighted screening at tau_dw (orc_jk_dw)."""
+    keep, args = _basis_args(sh, pure)
+    N = sh.nbf(pure)
+    D = np.ascontiguousarray(D, dtype=np.float64)
+    assert D.shape == (N, N)
+    J = np.zeros((N, N)); K = np.zeros((N, N))
+    Qp = None
+    if Q is not None:
+        Q = np.ascontiguousarray(Q, dtype=np.float64)
+        Qp = _d(Q)
+    _check(_get().orc_jk_dw(*args, _d(D), ctypes.c_double(tau), ctypes.c_double(tau_dw), Qp, _d(J), _d(K)), "jk_dw")
+    return J, K
+
+
 def jk_blocks(sh, D, pairs, tau=0.0, Q=None, pure=True):
     """Exact J/K blocks for shell pairs [(x, y), ...]: returns lists of [n_x, n_y] arrays."""
     keep, args = _basis_args(sh, pure)

@@ -39,7 +39,13 @@ struct Cls {
   static constexpr int KS1 = (NHAB + 3) / 4;  // GEMM1 k4 steps over p
   static constexpr int NT2 = (NCD + 7) / 8;   // GEMM2 n8 tiles over cd
   // register budget for the accumulators (doubles per lane): MC m-tiles per chunk
-  static constexpr int REGB = L >= 8 ? 56 : 40;
+#ifndef MAKO_REGB_HI
+#define MAKO_REGB_HI 56
+#endif
+#ifndef MAKO_REGB_LO
+#define MAKO_REGB_LO 40
+#endif
+  static constexpr int REGB = L >= 8 ? MAKO_REGB_HI : MAKO_REGB_LO;
   static constexpr int MCMAX = clampi(REGB / (2 * (NT1 + NT2)), 1, MT);
   static constexpr int NCHUNK = (MT + MCMAX - 1) / MCMAX;
   static constexpr int MC = (MT + NCHUNK - 1) / NCHUNK;

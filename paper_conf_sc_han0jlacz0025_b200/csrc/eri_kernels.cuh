@@ -44,19 +44,19 @@ constexpr int jk_minb() {
 
 // Persistent J/K kernel: each warp pulls tasks (bra pair, <= KT consecutive kets) from a global counter.
 // (An explicit minBlocks of 1 changes ptxas' register heuristic, so the cap is a separate wrapper.)
-template <int X, int Y>
+template <int X, int Y, bool DW>
 __device__ __forceinline__ void jk_body(const JKArgs& a);
-template <int X, int Y>
-__global__ void __launch_bounds__(CTA_THREADS) jk_kernel_free(JKArgs a) { jk_body<X, Y>(a); }
-template <int X, int Y>
-__global__ void __launch_bounds__(CTA_THREADS, 4) jk_kernel_capped(JKArgs a) { jk_body<X, Y>(a); }
-template <int X, int Y>
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(CTA_THREADS) jk_kernel_free(JKArgs a) { jk_body<X, Y, DW>(a); }
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(CTA_THREADS, 4) jk_kernel_capped(JKArgs a) { jk_body<X, Y, DW>(a); }
+template <int X, int Y, bool DW = false>
 constexpr auto jk_kernel_ptr() {
-  if constexpr (jk_minb<X, Y>() > 1) return &jk_kernel_capped<X, Y>;
-  else return &jk_kernel_free<X, Y>;
+  if constexpr (jk_minb<X, Y>() > 1) return &jk_kernel_capped<X, Y, DW>;
+  else return &jk_kernel_free<X, Y, DW>;
 }
 
-template <int X, int Y>
+template <int X, int Y, bool DW>
 __device__ __forceinline__ void jk_body(const JKArgs& a) {
   using C = ClsXY<X, Y>;
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -91,7 +91,7 @@ __device__ __forceinline__ void jk_body(const JKArgs& a) {
       const double QQ = QP * __ldg(a.ket.Q + R);
       if (QQ < a.thresh) continue;
       const int sc = __ldg(a.ket.shA + R), sd = __ldg(a.ket.shB + R);
-      if (!dw_keep(a, QQ, sa, sb, sc, sd)) continue;
+      if (!dw_keep<DW>(a, QQ, sa, sb, sc, sd)) continue;
       const int oc = __ldg(a.ao + sc), od = __ldg(a.ao + sd);
       d_prefetch<C>(jab + C::NAB, a.D, oa, ob, oc, od, a.nbf, lane);
       quartet_block<C>(a.bra, P, a.ket, R, Rbuf, V, htab, rtab, a.boys, lane);
@@ -209,16 +209,41 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   long long cap = (long long)nsm * bps / (a.grid_div > 1 ? a.grid_div : 1);
   if (cap < nsm) cap = nsm;
   const int grid = (int)(want < cap ? want : cap);
-  if constexpr (use_kf_swap<X, Y>())
-    kf_jk_kernel_ptr<Y, X>()<<<grid, CTA_THREADS, KfCfg<Y, X>::SMEM, (cudaStream_t)stream>>>(a);
-  else if constexpr (use_kf<X, Y>())
-    kf_jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
-  else if constexpr (use_tpq(X, Y))
-    tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, (cudaStream_t)stream>>>(a);
-  else if constexpr (use_slab<X, Y>())
-    slab_jk_kernel<X, Y><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, (cudaStream_t)stream>>>(a);
-  else
-    jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
+  // density-weighted screening (a.dsh != null) runs separate instantiations, so the plain build's
+  // kernels carry none of its code (it raised their register counts)
+  const cudaStream_t cs = (cudaStream_t)stream;
+  if constexpr (use_kf_swap<X, Y>()) {
+    if (a.dsh) {
+      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel_ptr<Y, X, true>(), KfCfg<Y, X>::SMEM)) return MAKO_ERR_CUDA;
+      kf_jk_kernel_ptr<Y, X, true>()<<<grid, CTA_THREADS, KfCfg<Y, X>::SMEM, cs>>>(a);
+    } else {
+      kf_jk_kernel_ptr<Y, X>()<<<grid, CTA_THREADS, KfCfg<Y, X>::SMEM, cs>>>(a);
+    }
+  } else if constexpr (use_kf<X, Y>()) {
+    if (a.dsh) {
+      if (set_smem_attr<X, Y>((const void*)kf_jk_kernel_ptr<X, Y, true>(), KfCfg<X, Y>::SMEM)) return MAKO_ERR_CUDA;
+      kf_jk_kernel_ptr<X, Y, true>()<<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, cs>>>(a);
+    } else {
+      kf_jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, cs>>>(a);
+    }
+  } else if constexpr (use_tpq(X, Y)) {
+    if (a.dsh) tpq_jk_kernel<X, Y, true><<<grid, CTA_THREADS, 0, cs>>>(a);
+    else tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, cs>>>(a);
+  } else if constexpr (use_slab<X, Y>()) {
+    if (a.dsh) {
+      if (set_smem_attr<X, Y>((const void*)slab_jk_kernel<X, Y, true>, SlabCfg<X, Y>::SMEM)) return MAKO_ERR_CUDA;
+      slab_jk_kernel<X, Y, true><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, cs>>>(a);
+    } else {
+      slab_jk_kernel<X, Y><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, cs>>>(a);
+    }
+  } else {
+    if (a.dsh) {
+      if (set_smem_attr<X, Y>((const void*)jk_kernel_ptr<X, Y, true>(), smem)) return MAKO_ERR_CUDA;
+      jk_kernel_ptr<X, Y, true>()<<<grid, CTA_THREADS, smem, cs>>>(a);
+    } else {
+      jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, smem, cs>>>(a);
+    }
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("jk_kernel launch: ") + cudaGetErrorString(e));
   if (nlaunch) ++*nlaunch;

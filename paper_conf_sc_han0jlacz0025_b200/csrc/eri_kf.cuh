@@ -64,19 +64,19 @@ constexpr bool use_kf_swap() {
   return false;
 }
 
-template <int X, int Y>
+template <int X, int Y, bool DW>
 __device__ __forceinline__ void kf_body(const JKArgs& a);
-template <int X, int Y>
-__global__ void __launch_bounds__(128) kf_kernel_free(JKArgs a) { kf_body<X, Y>(a); }
-template <int X, int Y>
-__global__ void __launch_bounds__(128, 3) kf_kernel_capped(JKArgs a) { kf_body<X, Y>(a); }
-template <int X, int Y>
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(128) kf_kernel_free(JKArgs a) { kf_body<X, Y, DW>(a); }
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(128, 3) kf_kernel_capped(JKArgs a) { kf_body<X, Y, DW>(a); }
+template <int X, int Y, bool DW = false>
 constexpr auto kf_jk_kernel_ptr() {
-  if constexpr (KfCfg<X, Y>::MINB > 1) return &kf_kernel_capped<X, Y>;
-  else return &kf_kernel_free<X, Y>;
+  if constexpr (KfCfg<X, Y>::MINB > 1) return &kf_kernel_capped<X, Y, DW>;
+  else return &kf_kernel_free<X, Y, DW>;
 }
 
-template <int X, int Y>
+template <int X, int Y, bool DW>
 __device__ __forceinline__ void kf_body(const JKArgs& a) {
   using C = ClsXY<X, Y>;
   using K = KfCfg<X, Y>;
@@ -110,7 +110,7 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
     const double QQ = QP * __ldg(a.ket.Q + min(R, r1 - 1));
     const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
     const bool active = R < r1 && QQ >= a.thresh &&
-                        dw_keep(a, QQ, sa, sb, __ldg(a.ket.shA + min(R, r1 - 1)), __ldg(a.ket.shB + min(R, r1 - 1)));
+                        dw_keep<DW>(a, QQ, sa, sb, __ldg(a.ket.shA + min(R, r1 - 1)), __ldg(a.ket.shB + min(R, r1 - 1)));
     const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
     const int b0 = __ldg(a.bra.poff + P), b1 = __ldg(a.bra.poff + P + 1);
     const int k0 = active ? __ldg(a.ket.poff + R) : 0, k1 = active ? __ldg(a.ket.poff + R + 1) : 0;

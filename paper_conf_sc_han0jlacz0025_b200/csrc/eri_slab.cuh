@@ -53,7 +53,7 @@ constexpr bool use_slab() {
   return !use_tpq(X, Y) && SlabCfg<X, Y>::OK && in_list(kSlabPick, X * 100 + Y);
 }
 
-template <int X, int Y>
+template <int X, int Y, bool DW = false>
 __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
   using C = ClsXY<X, Y>;
   using S = SlabCfg<X, Y>;
@@ -114,7 +114,7 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
       const bool cont = kl != __ldg(a.ket.poff + r);  // batch starts inside a ket (V row carries over)
       while (ns < nsl && r < r1) {
         const double QQ = QP * __ldg(a.ket.Q + r);
-        if (QQ < a.thresh || !dw_keep(a, QQ, sa, sb, __ldg(a.ket.shA + r), __ldg(a.ket.shB + r))) {
+        if (QQ < a.thresh || !dw_keep<DW>(a, QQ, sa, sb, __ldg(a.ket.shA + r), __ldg(a.ket.shB + r))) {
           ++r;
           if (r < r1) kl = __ldg(a.ket.poff + r);
           continue;

@@ -124,11 +124,15 @@ constexpr bool tpq_wacc() {
   return nH(C::L) + C::NAB * C::NCD + C::NHAB * C::NCD + C::NHCD * C::NCD <= 110;
 }
 
-constexpr int TASK_GRAB = 4;  // tasks taken per counter increment (one bra search per grab)
+#ifndef MAKO_TASK_GRAB
+#define MAKO_TASK_GRAB 4
+#endif
+constexpr int TASK_GRAB = MAKO_TASK_GRAB;  // tasks taken per counter increment (one entry lookup per grab)
 
 // density-weighted screening of quartet (sa sb|sc sd) with Schwarz product qq (reading R17)
+template <bool DW>
 __device__ __forceinline__ bool dw_keep(const JKArgs& a, double qq, int sa, int sb, int sc, int sd) {
-  if (a.dsh == nullptr) return true;
+  if constexpr (!DW) return true;
   const float* __restrict__ t = a.dsh;
   const size_t n = (size_t)a.nshell;
   const float m = fmaxf(fmaxf(__ldg(t + sa * n + sb), __ldg(t + sc * n + sd)),
@@ -150,7 +154,7 @@ __device__ __forceinline__ int find_entry(const JKArgs& a, long long task) {
 #else
 #define MAKO_TPQ_BOUNDS __launch_bounds__(128)
 #endif
-template <int X, int Y>
+template <int X, int Y, bool DW = false>
 __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
   using C = ClsXY<X, Y>;
   constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
@@ -175,7 +179,7 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
     const double QQ = QP * __ldg(a.ket.Q + min(R, r1 - 1));
     const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
     const bool active = R < r1 && QQ >= a.thresh &&
-                        dw_keep(a, QQ, sa, sb, __ldg(a.ket.shA + min(R, r1 - 1)), __ldg(a.ket.shB + min(R, r1 - 1)));
+                        dw_keep<DW>(a, QQ, sa, sb, __ldg(a.ket.shA + min(R, r1 - 1)), __ldg(a.ket.shB + min(R, r1 - 1)));
     const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
     const int b0 = __ldg(a.bra.poff + P), b1 = __ldg(a.bra.poff + P + 1);
     double V[NAB][NCD];

@@ -130,8 +130,12 @@ class Pairs:
     __del__ = close
 
 
-def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=None):
-    """J_{mn} = sum (mn|ls) D_ls, K_{ml} = sum (mn|ls) D_ns on the GPU (north_star).  Async on `stream`."""
+MAKO_JK_DENSITY_SCREEN = 1
+
+
+def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=None, density_screen=False):
+    """J_{mn} = sum (mn|ls) D_ls, K_{ml} = sum (mn|ls) D_ns on the GPU (north_star).  Async on `stream`
+    (density_screen=True: mako_build_jk_ex with MAKO_JK_DENSITY_SCREEN, which synchronises `stream`)."""
     n = pairs.basis.nbf
     if D.shape != (n, n):
         raise ValueError(f"D must be {n}x{n}")
@@ -139,8 +143,13 @@ def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=N
         J = torch.empty_like(D)
     if K is None:
         K = torch.empty_like(D)
-    check(pairs._lib.mako_build_jk(pairs.handle, _dev_ptr(D, "D"), float(pairs.tau if thresh is None else thresh),
-                                   _dev_ptr(J, "J"), _dev_ptr(K, "K"), int(shard), int(nshards), _stream_ptr(stream)))
+    t = float(pairs.tau if thresh is None else thresh)
+    if density_screen:
+        check(pairs._lib.mako_build_jk_ex(pairs.handle, _dev_ptr(D, "D"), t, MAKO_JK_DENSITY_SCREEN, _dev_ptr(J, "J"),
+                                          _dev_ptr(K, "K"), int(shard), int(nshards), _stream_ptr(stream)))
+    else:
+        check(pairs._lib.mako_build_jk(pairs.handle, _dev_ptr(D, "D"), t, _dev_ptr(J, "J"), _dev_ptr(K, "K"),
+                                       int(shard), int(nshards), _stream_ptr(stream)))
     return J, K
 
 

@@ -1,0 +1,117 @@
+"""GPU parity of density-weighted screening (mako_build_jk_ex, MAKO_JK_DENSITY_SCREEN) against the
+oracle's rule (orc_jk_dw), and of the incremental SCF against the
+plain SCF.  Bars: max|dJ|, max|dK| <= 1e-8; |dE_SCF| <= 1e-7 Ha (north_star)."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import mako_inputs as mi
+
+pytestmark = pytest.mark.gpu
+
+
+def _setup(cfg, tau):
+    from paper_conf_sc_han0jlacz0025_b200 import Basis, Pairs
+    m, b = mi.config_molecule(cfg)
+    sh = mi.shells_for(m, b)
+    B = Basis(m.Z, m.xyz_bohr, sh)
+    return m, sh, B, Pairs(B, tau)
+
+
+def _gpu(P, D, thresh, dw):
+    import torch
+    from paper_conf_sc_han0jlacz0025_b200 import build_jk
+    J, K = build_jk(P, torch.tensor(D, device="cuda"), thresh=thresh, density_screen=dw)
+    torch.cuda.synchronize()
+    return J.cpu().numpy(), K.cpu().numpy()
+
+
+def test_density_screen_vs_oracle_rule():
+    m, sh, B, P = _setup("benzene-def2svp", 1e-12)
+    Q = oracle.schwarz(sh)
+    for scale, tau_dw in ((1.0, 1e-9), (1e-3, 1e-9), (1e-6, 1e-10)):
+        D = mi.synthetic_density(sh.nbf(), m.nelec // 2, seed=4) * scale
+        J0, K0 = oracle.jk_dw(sh, D, 1e-12, tau_dw, Q=Q)
+        J, K = _gpu(P, D, tau_dw, True)
+        dj, dk = np.abs(J - J0).max(), np.abs(K - K0).max()
+        print("density screen", scale, tau_dw, dj, dk)
+        assert dj <= 1e-8 and dk <= 1e-8
+        assert np.array_equal(J, J.T) and np.array_equal(K, K.T)
+    # tau_dw -> 0: identical to the plain build
+    D = mi.synthetic_density(sh.nbf(), m.nelec // 2, seed=5)
+    J1, K1 = _gpu(P, D, 1e-12, False)
+    J2, K2 = _gpu(P, D, 1e-30, True)
+    assert np.abs(J1 - J2).max() <= 1e-12 * np.abs(J1).max() and np.abs(K1 - K2).max() <= 1e-12 * np.abs(K1).max()
+
+
+def _scf(mol, sh, jk_fn):
+    S, T, V = oracle.one_electron(sh, mol)
+    return oracle.rhf(S, T, V, oracle.nuclear_repulsion(mol), mol.nelec // 2, jk_fn)
+
+
+def test_incremental_scf_energies():
+    from paper_conf_sc_han0jlacz0025_b200 import Basis, IncrementalJK, Pairs
+    # published pin (tests/golden/h2o_sto3g.txt) through the incremental, density-screened GPU J/K
+    mol = mi.h2o_crawford()
+    sh = mi.shells_for(mol, "sto-3g")
+    P = Pairs(Basis(mol.Z, mol.xyz_bohr, sh), 1e-12)
+    inc = IncrementalJK(P)
+    r = _scf(mol, sh, inc)
+    assert r.converged and abs(r.energy - (-74.942079928192)) <= 1e-8
+    assert any(not h["full"] for h in inc.history)
+    # benzene: incremental vs plain GPU SCF and vs the oracle SCF
+    m, sh, B, P = _setup("benzene-def2svp", 1e-12)
+    inc = IncrementalJK(P)
+    r_inc = _scf(m, sh, inc)
+    r_gpu = _scf(m, sh, lambda D: _gpu(P, D, 1e-12, False))
+    r_orc = _scf(m, sh, lambda D: oracle.jk(sh, D, 1e-12))
+    print("benzene", r_inc.energy, r_gpu.energy, r_orc.energy, [(h["full"], h["tau"]) for h in inc.history])
+    assert r_inc.converged and abs(r_inc.energy - r_gpu.energy) <= 1e-7
+    assert abs(r_inc.energy - r_orc.energy) <= 1e-7
+    assert r_inc.iterations <= r_gpu.iterations + 4  # the schedule does not derail the SCF
+    hist = inc.history
+    assert hist[0]["full"] and not all(h["full"] for h in hist)
+    assert hist[-1]["tau"] == pytest.approx(1e-12)  # tightened to tau_final near convergence
+
+
+@pytest.mark.skipif(not os.environ.get("MAKO_SCF_TIMING"), reason="timing run (MAKO_SCF_TIMING=1)")
+def test_incremental_scf_timing():
+    """(Gly)10 def2-SVP RHF: per-iteration device time of plain vs incremental density-screened
+    J/K builds (the measurement of SURVEY S8.f row 2); written to gpurun_out/scf_timing.json."""
+    import time
+    import torch
+    from paper_conf_sc_han0jlacz0025_b200 import IncrementalJK, build_jk
+    m, sh, B, P = _setup(os.environ.get("MAKO_SCF_CONFIG", "gly10-def2svp"), 1e-12)
+    S, T, V = oracle.one_electron(sh, m)
+    enuc = oracle.nuclear_repulsion(m)
+    plain_ms = []
+
+    def plain(D):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        Dt = torch.tensor(D, device="cuda")
+        e0.record()
+        J, K = build_jk(P, Dt)
+        e1.record()
+        torch.cuda.synchronize()
+        plain_ms.append(e0.elapsed_time(e1))
+        return J.cpu().numpy(), K.cpu().numpy()
+
+    t0 = time.time()
+    r_plain = oracle.rhf(S, T, V, enuc, m.nelec // 2, plain, e_tol=1e-9, d_tol=1e-6)
+    t1 = time.time()
+    inc = IncrementalJK(P)
+    r_inc = oracle.rhf(S, T, V, enuc, m.nelec // 2, inc, e_tol=1e-9, d_tol=1e-6)
+    t2 = time.time()
+    out = {"config": os.environ.get("MAKO_SCF_CONFIG", "gly10-def2svp"), "nbf": sh.nbf(),
+           "plain": {"energy": r_plain.energy, "iterations": r_plain.iterations, "build_ms": plain_ms,
+                     "wall_s": t1 - t0},
+           "incremental": {"energy": r_inc.energy, "iterations": r_inc.iterations, "builds": inc.history,
+                           "wall_s": t2 - t1},
+           "dE": r_inc.energy - r_plain.energy}
+    os.makedirs("gpurun_out", exist_ok=True)
+    json.dump(out, open("gpurun_out/scf_timing.json", "w"), indent=1)
+    print(json.dumps({k: v for k, v in out.items() if k != "incremental"})[:500])
+    assert abs(r_inc.energy - r_plain.energy) <= 1e-7
