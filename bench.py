@@ -295,6 +295,40 @@ def run_mako(args):
         ms = float(t.item())
     value = flops_total / (ms * 1e-3) / 1e12
 
+    # stage-aware reduced-precision tier (mako_build_jk_mixed): same workload, quartets
+    # with Q_ab Q_cd max|D| < thresh_fp64 in the TF32 tier; error of the two-electron energy vs FP64
+    mixed = None
+    names_ = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff"]
+    if args.mixed > 0 and world == 1:
+        Jm, Km = torch.empty_like(D), torch.empty_like(D)
+        build_jk(P, D, J=Jm, K=Km, stream=stream, thresh_fp64=args.mixed)
+        torch.cuda.synchronize()
+        nm = max(1, min(args.steps, 3))
+        e0.record(stream)
+        for _ in range(nm):
+            build_jk(P, D, J=Jm, K=Km, stream=stream, thresh_fp64=args.mixed)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms_m = e0.elapsed_time(e1) / nm
+        cls_ms_m = None
+        if args.class_times:
+            P.profile(True)
+            build_jk(P, D, J=Jm, K=Km, stream=stream, thresh_fp64=args.mixed)
+            cls_ms_m, _ = P.profile_read()
+            P.profile(False)
+        e2 = lambda JJ, KK: 0.5 * float(torch.sum(D * (JJ - 0.5 * KK)))
+        mixed = {"thresh_fp64": args.mixed, "s_per_iter": ms_m * 1e-3, "value": flops_total / (ms_m * 1e-3) / 1e12,
+                 "unit": UNIT, "speedup_vs_fp64": ms / ms_m, "steps": nm,
+                 "dE2_vs_fp64_Ha": e2(Jm, Km) - e2(J, K),
+                 "max_dJ": float((Jm - J).abs().max()), "max_dK": float((Km - K).abs().max()),
+                 "tiers": "FP64 Boys/R + TF32 GEMM1/GEMM2 (FP32 accumulate) + FP64 digestion for quartets with "
+                          "Q_ab Q_cd max|D| < thresh_fp64 in the 31 classes with a reduced kernel; FP64 otherwise"}
+        if cls_ms_m is not None:
+            mixed["class_ms"] = {f"({names_[int((math.isqrt(8*i+1)-1)//2)]}|"
+                                 f"{names_[i - int((math.isqrt(8*i+1)-1)//2) * (int((math.isqrt(8*i+1)-1)//2) + 1) // 2]})":
+                                 round(float(cls_ms_m[i]), 4) for i in range(len(cls_ms_m)) if cls_ms_m[i] > 0}
+        del Jm, Km
+
     # end to end through the public API with host buffers (pinned), copies inside the timed region
     Dpin = torch.from_numpy(Dh).pin_memory()
     Jpin = torch.empty((n, n), dtype=torch.float64).pin_memory()
@@ -362,6 +396,8 @@ def run_mako(args):
             "clocks": clk, "roofline": roof,
             "e2e": {"value": flops_total / (ms_e2e * 1e-3) / 1e12, "unit": UNIT, "ms_per_step": ms_e2e,
                     "h2d_bytes_per_step": int(n * n * 8), "d2h_bytes_per_step": int(2 * n * n * 8)}}
+    if mixed is not None:
+        line["mixed_precision"] = mixed
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(sh, Dh, args.tau, flops_total, target_s=args.cpu_seconds)
     if args.class_times and rank == 0:
@@ -389,6 +425,8 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-step-s", type=float, default=6.0)
     ap.add_argument("--class-times", action="store_true")
+    ap.add_argument("--mixed", type=float, default=1e-6,
+                    help="thresh_fp64 of the reduced-precision measurement (0 = skip)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)

@@ -129,6 +129,27 @@ mako_status mako_build_jk(mako_pairs pairs, const double* D, double thresh, doub
 mako_status mako_build_jk_ex(mako_pairs pairs, const double* D, double thresh, unsigned flags, double* J, double* K,
                              int shard, int nshards, void* cuda_stream);
 
+/* Stage-aware reduced-precision J/K build (QuantMako, PAPER.md S3.2 L286-L302; SURVEY S8.f row 1;
+ * DESIGN.md readings R19-R20).  Three tiers per canonical quartet ("critical ones are
+ * evaluated with FP64 kernels, moderately important ones with quantized kernels, and negligible ones
+ * are pruned"):
+ *   Q_ab Q_cd < thresh (or the density rule of MAKO_JK_DENSITY_SCREEN)          pruned
+ *   Q_ab Q_cd max|D| < T, T = thresh_fp64 / max|D| rounded DOWN to a power of 10,
+ *     times max|D|  (i.e. a quartet whose J/K contribution bound is below ~thresh_fp64)
+ *                                                                                 reduced precision
+ *   otherwise                                                                      FP64
+ * max|D| is the global maximum |D_mn|.  The reduced tier keeps the Boys function and the R recursion
+ * in FP64, runs both Hermite->AO contractions (Eq. 7) as TF32 tensor-core GEMMs
+ * with FP32 accumulation (L296 first stage) and digests into FP64 J/K (L296 second stage).  Classes
+ * without a reduced-precision kernel (mako_class_reduced) run FP64 in both tiers.  Per-quartet error
+ * budget: |d(ab|cd)| <= (2^-9 + (K1+K2) 2^-24) * sum|E~ R E~| (eri_quant.cuh).  thresh_fp64 > 0
+ * (finite); thresh as in mako_build_jk_ex; flags: 0 or MAKO_JK_DENSITY_SCREEN.  SYNCHRONISES
+ * cuda_stream once (max|D| decides the tier plan).  D, J, K as in mako_build_jk. */
+mako_status mako_build_jk_mixed(mako_pairs pairs, const double* D, double thresh, double thresh_fp64,
+                                unsigned flags, double* J, double* K, int shard, int nshards, void* cuda_stream);
+/* mask[MAKO_NCLASS] (HOST): 1 where the class has a reduced-precision (TF32) kernel. */
+mako_status mako_class_reduced(int* mask);
+
 /* Number of CUDA kernels one mako_build_jk call launches for these arguments (for bench accounting). */
 mako_status mako_build_jk_launches(mako_pairs pairs, double thresh, int shard, int nshards, int* n_launches);
 
@@ -156,6 +177,12 @@ mako_status mako_profile_read(mako_pairs pairs, double* ms, long long* launches)
  * (the temporary pair data is freed). */
 mako_status mako_eri_batch(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,
                            void* cuda_stream);
+/* As mako_eri_batch; flags = MAKO_ERI_REDUCED evaluates the quartets of classes that have a
+ * reduced-precision kernel with it (the tier mako_build_jk_mixed uses; for its error budget and RMSE,
+ * PAPER.md Table 2).  flags = 0 is exactly mako_eri_batch. */
+#define MAKO_ERI_REDUCED 1u
+mako_status mako_eri_batch_ex(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,
+                              unsigned flags, void* cuda_stream);
 
 /* Boys function F_m(T), m = 0..mmax (mmax <= 4*MAKO_LMAX), for n values T[n] (DEVICE pointers),
  * out[n*(mmax+1)] (DEVICE).  Exposes the device Boys evaluator of the hot path for parity tests. */

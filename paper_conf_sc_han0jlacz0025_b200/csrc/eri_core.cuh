@@ -196,11 +196,19 @@ __device__ __forceinline__ void boys_eval(double T, const double* __restrict__ t
 //   R^{(n)}_{000} = (-2 rho)^n F_n(rho |PQ|^2) * 2 pi^{5/2} / sqrt(p+q)
 //   R^{(n)}_{t+1,u,v} = t R^{(n+1)}_{t-1,u,v} + X_PQ R^{(n+1)}_{t,u,v}   (and u, v alike)
 // Level n holds all entries with t+u+v <= L-n; lanes split each level; levels ping-pong.
-template <class C>
+// F32: level 0 is written TF32-rounded into dst32 instead of dst (reduced-precision tier, eri_quant.cuh;
+// the recursion itself stays FP64)
+__device__ __forceinline__ float to_tf32(double x) {
+  unsigned r;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"((float)x));
+  return __uint_as_float(r);
+}
+
+template <class C, bool F32 = false>
 __device__ __forceinline__ void compute_R(double p, double Px, double Py, double Pz, double q, double Qx, double Qy,
                                           double Qz, double* __restrict__ dst, double* __restrict__ scratch,
                                           const uint32_t* __restrict__ rtab, const double* __restrict__ btab,
-                                          int lane) {
+                                          int lane, float* __restrict__ dst32 = nullptr) {
   constexpr int L = C::L, NH = C::NH;
   const double pq = p + q, ri = rsqrt_fast(pq), rho = p * q * ri * ri;
   const double X = Px - Qx, Y = Py - Qy, Z = Pz - Qz;
@@ -215,7 +223,10 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
     s *= m2r;
   }
   if constexpr (L == 0) {
-    if (lane == 0) dst[0] = F[0];
+    if (lane == 0) {
+      if constexpr (F32) dst32[0] = to_tf32(F[0]);
+      else dst[0] = F[0];
+    }
     __syncwarp();
   } else {
     if (lane == 0) ((L & 1) ? scratch : dst)[0] = F[L];
@@ -236,7 +247,8 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
           v = xd * prv[s1];
           if (cf) v = fma((double)cf, prv[s2], v);
         }
-        cur[e] = v;
+        if (F32 && n == 0) dst32[e] = to_tf32(v);
+        else cur[e] = v;
       }
       __syncwarp();
     }

@@ -20,16 +20,29 @@ template <int X, int Y>
 int task_kets_xy();
 template <int X, int Y>
 bool swap_xy();
+template <int X, int Y>
+bool lowp_xy();
 
 }  // namespace mako
 
 #ifdef MAKO_DEFINE_KERNELS
+#include <algorithm>
+
 #include "eri_core.cuh"
 #include "eri_tpq.cuh"
 #include "eri_slab.cuh"
 #include "eri_kf.cuh"
+#include "eri_quant.cuh"
 
 namespace mako {
+
+// classes with a reduced-precision (TF32) tier kernel: the warp-per-quartet DMMA family, where the
+// basis transformation (GEMM1/GEMM2) dominates (the lane-per-ket, ket-first and
+// slab families run the FP64 kernel in both tiers)
+template <int X, int Y>
+constexpr bool has_lowp() {
+  return !use_tpq(X, Y) && !use_kf<X, Y>() && !use_kf_swap<X, Y>() && !use_slab<X, Y>();
+}
 
 template <class C>
 __host__ __device__ constexpr size_t cta_smem_bytes() {
@@ -109,6 +122,111 @@ __device__ __forceinline__ void jk_body(const JKArgs& a) {
   }
 }
 
+// eri_batch store epilogue: canonical V[A][B][C][D] -> user order [a][b][c][d] (undo the swaps)
+template <class C>
+__device__ void store_block(const BatchArgs& a, int qi, const double* __restrict__ V, int lane) {
+  const int fl = a.qflag[qi];
+  const bool sab = fl & 1, scd = fl & 2, sbk = fl & 4;
+  const int n[4] = {C::NA, C::NB, C::NC, C::ND};
+  // user positions of the canonical shells A, B, C, D, and the sizes in user order
+  const int posA = sbk ? (scd ? 3 : 2) : (sab ? 1 : 0);
+  const int posB = sbk ? (scd ? 2 : 3) : (sab ? 0 : 1);
+  const int posC = sbk ? (sab ? 1 : 0) : (scd ? 3 : 2);
+  const int posD = sbk ? (sab ? 0 : 1) : (scd ? 2 : 3);
+  int nu[4];
+  nu[posA] = n[0]; nu[posB] = n[1]; nu[posC] = n[2]; nu[posD] = n[3];
+  const size_t base = (size_t)a.qout[qi];
+  for (int e = lane; e < C::NAB * C::NCD; e += 32) {
+    int idx[4];
+    const int ab = e / C::NCD, cd = e % C::NCD;
+    idx[posA] = ab / C::NB; idx[posB] = ab % C::NB; idx[posC] = cd / C::ND; idx[posD] = cd % C::ND;
+    a.out[base + (((size_t)idx[0] * nu[1] + idx[1]) * nu[2] + idx[2]) * nu[3] + idx[3]] = V[e];
+  }
+}
+
+// Reduced-precision tier of the persistent J/K kernel (eri_quant.cuh): the task loop and the FP64
+// digestion of jk_body, the TF32 basis transformation of quartet_block_q.
+template <class C>
+__host__ __device__ constexpr size_t cta_smem_bytes_q() {
+  return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)CTA_WARPS * ClsQ<C>::WARP_DBL;
+}
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(CTA_THREADS) jk_kernel_q(JKArgs a) {
+  using C = ClsXY<X, Y>;
+  using Q = ClsQ<C>;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  uint16_t* htab = reinterpret_cast<uint16_t*>(smem_raw);
+  uint32_t* rtab = reinterpret_cast<uint32_t*>(smem_raw + C::HTAB_BYTES);
+  double* wbase = reinterpret_cast<double*>(smem_raw + C::HTAB_BYTES + C::RTAB_BYTES);
+  init_tables<C>(htab, rtab);
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  double* Rbuf = wbase + (size_t)warp * Q::WARP_DBL;
+  double* V = Rbuf + C::W_R;
+  double* jab = V + C::W_V;
+  float* R32 = reinterpret_cast<float*>(Rbuf + C::WARP_DBL);
+  for (;;) {
+  unsigned long long grab = 0;
+  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
+  grab = __shfl_sync(0xffffffffu, grab, 0);
+  const long long tg0 = a.task_begin + (long long)grab;
+  if (tg0 >= a.task_end) break;
+  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  int U = find_entry(a, tg0);
+  for (long long task = tg0; task < tg1; ++task) {
+    while (__ldg(a.task_off + U + 1) <= task) ++U;
+    const int P = __ldg(a.ent_P + U);
+    const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * a.KT;
+    const int r1 = min(r0 + a.KT, __ldg(a.kend + U));
+    const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
+    const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
+    const double QP = __ldg(a.bra.Q + P);
+    for (int i = lane; i < C::NAB; i += 32) jab[i] = 0.0;
+    __syncwarp();
+    for (int R = r0; R < r1; ++R) {
+      const double QQ = QP * __ldg(a.ket.Q + R);
+      if (QQ < a.thresh) continue;
+      const int sc = __ldg(a.ket.shA + R), sd = __ldg(a.ket.shB + R);
+      if (!dw_keep<DW>(a, QQ, sa, sb, sc, sd)) continue;
+      const int oc = __ldg(a.ao + sc), od = __ldg(a.ao + sd);
+      d_prefetch<C>(jab + C::NAB, a.D, oa, ob, oc, od, a.nbf, lane);
+      quartet_block_q<C>(a.bra, P, a.ket, R, Rbuf, R32, V, htab, rtab, a.boys, lane);
+      double deg = 1.0;
+      if (sa == sb) deg *= 0.5;
+      if (sc == sd) deg *= 0.5;
+      if (a.same_bucket && P == R) deg *= 0.5;
+      digest<C, false>(V, deg, oa, ob, oc, od, a.D, a.nbf, a.J, a.K, jab, jab + C::NAB, Rbuf, lane);
+      __syncwarp();
+    }
+    for (int ab = lane; ab < C::NAB; ab += 32)
+      atomicAdd(a.J + (size_t)(oa + ab / C::NB) * a.nbf + ob + ab % C::NB, jab[ab]);
+    __syncwarp();
+  }
+  }
+}
+
+// TF32-tier batch kernel (store epilogue only): eri_batch with MAKO_ERI_REDUCED
+template <int X, int Y>
+__global__ void __launch_bounds__(CTA_THREADS) batch_kernel_q(BatchArgs a) {
+  using C = ClsXY<X, Y>;
+  using Q = ClsQ<C>;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  uint16_t* htab = reinterpret_cast<uint16_t*>(smem_raw);
+  uint32_t* rtab = reinterpret_cast<uint32_t*>(smem_raw + C::HTAB_BYTES);
+  double* wbase = reinterpret_cast<double*>(smem_raw + C::HTAB_BYTES + C::RTAB_BYTES);
+  init_tables<C>(htab, rtab);
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  double* Rbuf = wbase + (size_t)warp * Q::WARP_DBL;
+  double* V = Rbuf + C::W_R;
+  float* R32 = reinterpret_cast<float*>(Rbuf + C::WARP_DBL);
+  for (int qi = blockIdx.x * CTA_WARPS + warp; qi < a.nq; qi += gridDim.x * CTA_WARPS) {
+    quartet_block_q<C>(a.bra, a.qbra[qi], a.ket, a.qket[qi], Rbuf, R32, V, htab, rtab, a.boys, lane);
+    store_block<C>(a, qi, V, lane);
+    __syncwarp();
+  }
+}
+
 // Batch kernel: one warp per listed quartet; store (eri_batch) or Schwarz-diagonal epilogue.
 template <int X, int Y>
 __global__ void __launch_bounds__(CTA_THREADS) batch_kernel(BatchArgs a) {
@@ -132,27 +250,7 @@ __global__ void __launch_bounds__(CTA_THREADS) batch_kernel(BatchArgs a) {
       for (int o = 16; o > 0; o >>= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
       if (lane == 0) a.out[a.qout[qi]] = sqrt(m);
     } else {
-      // canonical V[A][B][C][D] -> user order [a][b][c][d] (undo the swaps)
-      const int fl = a.qflag[qi];
-      const bool sab = fl & 1, scd = fl & 2, sbk = fl & 4;
-      int n[4] = {C::NA, C::NB, C::NC, C::ND};
-      // sizes in user order
-      int nu[4];
-      {
-        // user positions of the canonical shells A, B, C, D
-        int posA = sbk ? (scd ? 3 : 2) : (sab ? 1 : 0);
-        int posB = sbk ? (scd ? 2 : 3) : (sab ? 0 : 1);
-        int posC = sbk ? (sab ? 1 : 0) : (scd ? 3 : 2);
-        int posD = sbk ? (sab ? 0 : 1) : (scd ? 2 : 3);
-        nu[posA] = n[0]; nu[posB] = n[1]; nu[posC] = n[2]; nu[posD] = n[3];
-        const size_t base = (size_t)a.qout[qi];
-        for (int e = lane; e < C::NAB * C::NCD; e += 32) {
-          int idx[4];
-          int ab = e / C::NCD, cd = e % C::NCD;
-          idx[posA] = ab / C::NB; idx[posB] = ab % C::NB; idx[posC] = cd / C::ND; idx[posD] = cd % C::ND;
-          a.out[base + (((size_t)idx[0] * nu[1] + idx[1]) * nu[2] + idx[2]) * nu[3] + idx[3]] = V[e];
-        }
-      }
+      store_block<C>(a, qi, V, lane);
     }
     __syncwarp();
   }
@@ -212,6 +310,27 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   // density-weighted screening (a.dsh != null) runs separate instantiations, so the plain build's
   // kernels carry none of its code (it raised their register counts)
   const cudaStream_t cs = (cudaStream_t)stream;
+  if constexpr (has_lowp<X, Y>()) {
+    if (a.lowp) {
+      constexpr size_t sq = cta_smem_bytes_q<C>();
+      // the TF32 tier's own occupancy (its SMEM is larger by the TF32 R rows)
+      static int bq = -1;
+      if (bq < 0) {
+        if (set_smem_attr<X, Y>((const void*)jk_kernel_q<X, Y>, sq) ||
+            set_smem_attr<X, Y>((const void*)jk_kernel_q<X, Y, true>, sq))
+          return MAKO_ERR_CUDA;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bq, jk_kernel_q<X, Y>, CTA_THREADS, sq);
+        if (bq < 1) bq = 1;
+      }
+      const long long gq = std::min<long long>(want, std::max<long long>((long long)nsm * bq, nsm));
+      if (a.dsh) jk_kernel_q<X, Y, true><<<(int)gq, CTA_THREADS, sq, cs>>>(a);
+      else jk_kernel_q<X, Y><<<(int)gq, CTA_THREADS, sq, cs>>>(a);
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("jk_kernel_q launch: ") + cudaGetErrorString(e));
+      if (nlaunch) ++*nlaunch;
+      return MAKO_OK;
+    }
+  }
   if constexpr (use_kf_swap<X, Y>()) {
     if (a.dsh) {
       if (set_smem_attr<X, Y>((const void*)kf_jk_kernel_ptr<Y, X, true>(), KfCfg<Y, X>::SMEM)) return MAKO_ERR_CUDA;
@@ -255,10 +374,21 @@ mako_status launch_batch_xy(const BatchArgs& a, void* stream) {
   using C = ClsXY<X, Y>;
   constexpr size_t smem = cta_smem_bytes<C>();
   if (a.nq <= 0) return MAKO_OK;
-  mako_status st = set_smem_attr<X, Y>((const void*)batch_kernel<X, Y>, smem);
-  if (st) return st;
   int grid = (a.nq + CTA_WARPS - 1) / CTA_WARPS;
   if (grid > 148 * 64) grid = 148 * 64;
+  if constexpr (has_lowp<X, Y>()) {
+    if (a.lowp && !a.diag) {
+      constexpr size_t sq = cta_smem_bytes_q<C>();
+      mako_status st = set_smem_attr<X, Y>((const void*)batch_kernel_q<X, Y>, sq);
+      if (st) return st;
+      batch_kernel_q<X, Y><<<grid, CTA_THREADS, sq, (cudaStream_t)stream>>>(a);
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("batch_kernel_q launch: ") + cudaGetErrorString(e));
+      return MAKO_OK;
+    }
+  }
+  mako_status st = set_smem_attr<X, Y>((const void*)batch_kernel<X, Y>, smem);
+  if (st) return st;
   batch_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("batch_kernel launch: ") + cudaGetErrorString(e));
@@ -279,6 +409,10 @@ template <int X, int Y>
 bool swap_xy() {
   return use_kf_swap<X, Y>();
 }
+template <int X, int Y>
+bool lowp_xy() {
+  return has_lowp<X, Y>();
+}
 }  // namespace mako
 
 #define MAKO_INSTANTIATE(X, Y)                                                                   \
@@ -286,5 +420,6 @@ bool swap_xy() {
   template mako_status mako::launch_batch_xy<X, Y>(const mako::BatchArgs&, void*);               \
   template int mako::jk_blocks_per_sm<X, Y>();                                                   \
   template int mako::task_kets_xy<X, Y>();                                                       \
-  template bool mako::swap_xy<X, Y>();
+  template bool mako::swap_xy<X, Y>();                                                            \
+  template bool mako::lowp_xy<X, Y>();
 #endif

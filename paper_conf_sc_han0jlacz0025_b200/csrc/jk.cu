@@ -7,6 +7,7 @@
 // Sharding: shard s of n takes tasks [T s/n, T (s+1)/n) of every class.
 #include <algorithm>
 #include <cmath>
+#include <limits>
 
 #include "eri_kernels.cuh"
 #include "eri_core.cuh"
@@ -53,6 +54,14 @@ static bool class_swap(int X, int Y) {
   return false;
 }
 
+bool class_has_lowp(int X, int Y) {
+#define MAKO_LP_CASE(x, y) \
+  if (X == x && Y == y) return lowp_xy<x, y>();
+  MAKO_CLASS_LIST(MAKO_LP_CASE)
+#undef MAKO_LP_CASE
+  return false;
+}
+
 static mako_status cuda_check(cudaError_t e, const char* what) {
   if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
   return MAKO_OK;
@@ -76,10 +85,56 @@ static int prefix_count(const std::vector<double>& QY, int lo0, int hi0, double 
   return lo - lo0;
 }
 
-static mako_status ensure_plan(mako_pairs P, double thresh) {
-  if (P->plan.thresh == thresh && !P->plan.cls.empty()) return MAKO_OK;
+// entries of class plan c for the kets with lo <= Q_P Q_R < hi (hi = +inf: the plain Schwarz prefix);
+// in a Q-sorted segment that is the range [prefix(hi), prefix(lo)) of the segment
+static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const PairBucket& by, bool same, double lo,
+                                    double hi) {
+  const int nbra = bx.n(), G = NKGROUP;
+  c.ent_P.clear();
+  c.kbeg.clear();
+  c.kend.clear();
+  c.task_off.assign(1, 0);
+  c.nquartet = 0;
+  for (int p = 0; p < nbra; ++p)
+    for (int g = 0; g < G; ++g) {
+      const int s0 = by.seg.empty() ? 0 : by.seg[g], s1 = by.seg.empty() ? (g == 0 ? by.n() : 0) : by.seg[g + 1];
+      if (s1 <= s0) continue;
+      int nk = prefix_count(by.Q, s0, s1, bx.Q[p], lo);
+      int nh = std::isinf(hi) ? 0 : prefix_count(by.Q, s0, s1, bx.Q[p], hi);
+      if (same) {  // canonical: ket position <= bra position
+        nk = std::min(nk, std::max(0, p - s0 + 1));
+        nh = std::min(nh, nk);
+      }
+      if (nk <= nh) continue;
+      c.ent_P.push_back(p);
+      c.kbeg.push_back(s0 + nh);
+      c.kend.push_back(s0 + nk);
+      c.nquartet += nk - nh;
+      c.task_off.push_back(c.task_off.back() + (nk - nh + c.KT - 1) / c.KT);
+    }
+  c.ntask = c.task_off.back();
+  c.usamp.assign((size_t)(c.ntask >> TASK_SAMPLE_SHIFT) + 1, 0);
+  for (size_t u = 0, k = 0; k < c.usamp.size(); ++k) {
+    const long long t = (long long)k << TASK_SAMPLE_SHIFT;
+    while (u + 1 < c.ent_P.size() && c.task_off[u + 1] <= t) ++u;
+    c.usamp[k] = (int)u;
+  }
+  mako_status st;
+  if (c.ntask > 0 && ((st = upload(c.d_kbeg, c.kbeg)) || (st = upload(c.d_kend, c.kend)) ||
+                      (st = upload(c.d_task_off, c.task_off)) || (st = upload(c.d_ent_P, c.ent_P)) ||
+                      (st = upload(c.d_usamp, c.usamp))))
+    return st;
+  return MAKO_OK;
+}
+
+// Plan for Schwarz threshold `thresh`; with tier > thresh (reduced-precision build)
+// the quartets of classes that have a TF32-tier kernel are split: Q_ab Q_cd >= tier into cls (FP64),
+// thresh <= Q_ab Q_cd < tier into cls_lo (TF32).  tier = 0: one FP64 tier.
+static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0) {
+  if (!(tier > thresh)) tier = 0.0;
+  if (P->plan.thresh == thresh && P->plan.tier == tier && !P->plan.cls.empty()) return MAKO_OK;
   for (auto& sp : P->plan_cache)
-    if (sp.thresh == thresh && !sp.cls.empty()) {
+    if (sp.thresh == thresh && sp.tier == tier && !sp.cls.empty()) {
       std::swap(P->plan, sp);
       return MAKO_OK;
     }
@@ -89,51 +144,30 @@ static mako_status ensure_plan(mako_pairs P, double thresh) {
   }
   P->plan = Plan();
   Plan& pl = P->plan;
-  pl.cls.clear();
-  pl.cls.resize(NBUCKET * (NBUCKET + 1) / 2);
+  const int NCL = NBUCKET * (NBUCKET + 1) / 2;
+  pl.cls.resize(NCL);
+  pl.cls_lo.resize(NCL);
   pl.KT = 16;
+  const double inf = std::numeric_limits<double>::infinity();
   for (int X = 0; X < NBUCKET; ++X)
     for (int Y = 0; Y <= X; ++Y) {
-      ClassPlan& c = pl.cls[class_index(X, Y)];
-      c.X = X;
-      c.Y = Y;
-      c.KT = class_task_kets(X, Y);
-      c.swap = class_swap(X, Y);
-      c.TB = c.swap ? Y : X;
-      c.LB = c.swap ? X : Y;
-      const PairBucket& bx = P->set.b[c.TB];
-      const PairBucket& by = P->set.b[c.LB];
-      const int nbra = bx.n(), G = NKGROUP;
-      c.ent_P.clear();
-      c.kbeg.clear();
-      c.kend.clear();
-      c.task_off.assign(1, 0);
-      for (int p = 0; p < nbra; ++p)
-        for (int g = 0; g < G; ++g) {
-          const int s0 = by.seg.empty() ? 0 : by.seg[g], s1 = by.seg.empty() ? (g == 0 ? by.n() : 0) : by.seg[g + 1];
-          int nk = s1 > s0 ? prefix_count(by.Q, s0, s1, bx.Q[p], thresh) : 0;
-          if (X == Y) nk = std::min(nk, std::max(0, p - s0 + 1));  // canonical: ket position <= bra position
-          if (nk <= 0) continue;
-          c.ent_P.push_back(p);
-          c.kbeg.push_back(s0);
-          c.kend.push_back(s0 + nk);
-          c.nquartet += nk;
-          c.task_off.push_back(c.task_off.back() + (nk + c.KT - 1) / c.KT);
-        }
-      c.ntask = c.task_off.back();
-      c.usamp.assign((size_t)(c.ntask >> TASK_SAMPLE_SHIFT) + 1, 0);
-      for (size_t u = 0, k = 0; k < c.usamp.size(); ++k) {
-        const long long t = (long long)k << TASK_SAMPLE_SHIFT;
-        while (u + 1 < c.ent_P.size() && c.task_off[u + 1] <= t) ++u;
-        c.usamp[k] = (int)u;
+      const int ci = class_index(X, Y);
+      const bool split = tier > 0.0 && class_has_lowp(X, Y);
+      for (int part = 0; part < (split ? 2 : 1); ++part) {
+        ClassPlan& c = part ? pl.cls_lo[ci] : pl.cls[ci];
+        c.X = X;
+        c.Y = Y;
+        c.KT = class_task_kets(X, Y);
+        c.swap = class_swap(X, Y);
+        c.TB = c.swap ? Y : X;
+        c.LB = c.swap ? X : Y;
+        const double lo = part ? thresh : (split ? tier : thresh), hi = part ? tier : inf;
+        mako_status st = build_class_plan(c, P->set.b[c.TB], P->set.b[c.LB], X == Y, lo, hi);
+        if (st) return st;
       }
-      mako_status st;
-      if (c.ntask > 0 && ((st = upload(c.d_kbeg, c.kbeg)) || (st = upload(c.d_kend, c.kend)) ||
-                          (st = upload(c.d_task_off, c.task_off)) || (st = upload(c.d_ent_P, c.ent_P)) ||
-                          (st = upload(c.d_usamp, c.usamp))))
-        return st;
     }
   pl.thresh = thresh;
+  pl.tier = tier;
   return MAKO_OK;
 }
 
@@ -382,8 +416,10 @@ extern "C" mako_status mako_build_jk_launches(mako_pairs p, double thresh, int s
   return MAKO_OK;
 }
 
-static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, unsigned flags, double* J, double* K,
-                                 int shard, int nshards, void* cuda_stream) {
+// tier > 0 (mako_build_jk_mixed): quartets with Q_ab Q_cd max|D| >= tier stay FP64, the rest of the
+// classes that have a TF32-tier kernel run it (§3.2.3)
+static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, double tier, unsigned flags, double* J,
+                                 double* K, int shard, int nshards, void* cuda_stream) {
   try {
     mako_status st;
     if ((st = check_pairs(p))) return st;
@@ -395,9 +431,11 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, u
     const mako_basis_s* B = p->basis;
     const int n = B->nbf;
     cudaStream_t s = (cudaStream_t)cuda_stream;
+    if (!(tier >= 0) || !std::isfinite(tier)) return fail(MAKO_ERR_INVALID, "thresh_fp64 must be finite and >= 0");
     const bool dw = (flags & MAKO_JK_DENSITY_SCREEN) != 0;
     const double dw_thresh = std::max(thresh, p->tau);
-    if (dw) {
+    double tier_plan = 0.0;
+    if (dw || tier > 0) {
       // shell-block maxima of |D| and the global max; the task plan is the Schwarz prefix at
       // thresh / max|D| rounded down to a power of ten (a superset of the density-screened quartets,
       // few distinct plans over an SCF run), each quartet is then tested in the kernels
@@ -412,13 +450,18 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, u
           (st = cuda_check(cudaStreamSynchronize(s), "dmax sync")))
         return st;
       if (!std::isfinite(dmax)) return fail(MAKO_ERR_INVALID, "D is not finite");
-      thresh = dmax > 0 ? std::pow(10.0, std::floor(std::log10(dw_thresh / dmax))) : 1e300;
+      if (dw) thresh = dmax > 0 ? std::pow(10.0, std::floor(std::log10(dw_thresh / dmax))) : 1e300;
+      // tier boundary on Q_ab Q_cd: tier / max|D| rounded down to a power of ten (more FP64 work, few
+      // distinct plans over an SCF run)
+      if (tier > 0) tier_plan = dmax > 0 ? std::pow(10.0, std::floor(std::log10(tier / dmax))) : 0.0;
     }
     thresh = std::max(thresh, p->tau);
-    if ((st = ensure_plan(p, thresh))) return st;
+    if ((st = ensure_plan(p, thresh, tier_plan))) return st;
+    const bool mixed = p->plan.tier > 0.0;
+    if (mixed && (st = ensure_lowp(p->set, cuda_stream))) return st;
     if ((st = cuda_check(cudaMemsetAsync(J, 0, sizeof(double) * n * n, s), "memset J")) ||
         (st = cuda_check(cudaMemsetAsync(K, 0, sizeof(double) * n * n, s), "memset K")) ||
-        (st = cuda_check(cudaMemsetAsync(p->d_counters.p, 0, sizeof(unsigned long long) * 64, s), "memset ctr")))
+        (st = cuda_check(cudaMemsetAsync(p->d_counters.p, 0, sizeof(unsigned long long) * 128, s), "memset ctr")))
       return st;
     int nl = 0;
     if ((st = ensure_streams(p))) return st;
@@ -427,17 +470,21 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, u
     for (void* is : p->streams) cudaStreamWaitEvent((cudaStream_t)is, (cudaEvent_t)p->ev_fork, 0);
     // classes in descending estimated cost, greedily balanced over the internal streams; each kernel
     // gets half of the resident capacity so two classes (often a DFMA- and a DMMA-bound one) co-reside
+    // (index >= 55: the class's TF32-tier plan)
+    const int NCL = (int)p->plan.cls.size();
     std::vector<std::pair<double, int>> order;
-    for (size_t i = 0; i < p->plan.cls.size(); ++i) {
-      const ClassPlan& c = p->plan.cls[i];
+    for (int i = 0; i < (mixed ? 2 * NCL : NCL); ++i) {
+      const ClassPlan& c = i < NCL ? p->plan.cls[i] : p->plan.cls_lo[i - NCL];
+      if (c.ntask == 0) continue;
       const double cost = (double)c.nquartet * (nsph(bucket_la(c.X)) * nsph(bucket_lb(c.X)) *
                                                     nsph(bucket_la(c.Y)) * nsph(bucket_lb(c.Y)) + 16.0);
-      order.push_back({-cost, (int)i});
+      order.push_back({-cost, i});
     }
     std::sort(order.begin(), order.end());
     std::vector<double> load(p->streams.size(), 0.0);
     for (auto& oc : order) {
-      ClassPlan& c = p->plan.cls[oc.second];
+      const bool lo = oc.second >= NCL;
+      ClassPlan& c = lo ? p->plan.cls_lo[oc.second - NCL] : p->plan.cls[oc.second];
       JKArgs a{};
       a.task_begin = c.ntask * shard / nshards;
       a.task_end = c.ntask * (shard + 1) / nshards;
@@ -455,7 +502,7 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, u
       a.usamp = c.d_usamp.as<int>();
       a.nent = (int)c.kbeg.size();
       a.KT = c.KT;
-      a.counter = p->d_counters.as<unsigned long long>() + class_index(c.X, c.Y);
+      a.counter = p->d_counters.as<unsigned long long>() + class_index(c.X, c.Y) + (lo ? NCL : 0);
       a.D = D;
       a.J = J;
       a.K = K;
@@ -467,6 +514,7 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, u
       a.dw_thresh = dw_thresh;
       a.boys = B->d_boys.as<double>();
       a.grid_div = 1;
+      a.lowp = lo ? 1 : 0;
       cudaEvent_t e0 = nullptr, e1 = nullptr;
       if (p->prof) {
         cudaEventCreate(&e0);
@@ -493,17 +541,32 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, u
 
 extern "C" mako_status mako_build_jk(mako_pairs p, const double* D, double thresh, double* J, double* K, int shard,
                                      int nshards, void* cuda_stream) {
-  return build_jk_impl(p, D, thresh, 0u, J, K, shard, nshards, cuda_stream);
+  return build_jk_impl(p, D, thresh, 0.0, 0u, J, K, shard, nshards, cuda_stream);
 }
 
 extern "C" mako_status mako_build_jk_ex(mako_pairs p, const double* D, double thresh, unsigned flags, double* J,
                                         double* K, int shard, int nshards, void* cuda_stream) {
-  return build_jk_impl(p, D, thresh, flags, J, K, shard, nshards, cuda_stream);
+  return build_jk_impl(p, D, thresh, 0.0, flags, J, K, shard, nshards, cuda_stream);
 }
 
-extern "C" mako_status mako_eri_batch(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,
-                                      void* cuda_stream) {
+extern "C" mako_status mako_build_jk_mixed(mako_pairs p, const double* D, double thresh, double thresh_fp64,
+                                           unsigned flags, double* J, double* K, int shard, int nshards,
+                                           void* cuda_stream) {
+  if (!(thresh_fp64 > 0) || !std::isfinite(thresh_fp64)) return fail(MAKO_ERR_INVALID, "thresh_fp64 must be > 0");
+  return build_jk_impl(p, D, thresh, thresh_fp64, flags, J, K, shard, nshards, cuda_stream);
+}
+
+extern "C" mako_status mako_class_reduced(int* mask) {
+  if (!mask) return fail(MAKO_ERR_INVALID, "NULL mask");
+  for (int X = 0; X < NBUCKET; ++X)
+    for (int Y = 0; Y <= X; ++Y) mask[class_index(X, Y)] = class_has_lowp(X, Y) ? 1 : 0;
+  return MAKO_OK;
+}
+
+static mako_status eri_batch_impl(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,
+                                  unsigned flags, void* cuda_stream) {
   try {
+    if (flags & ~(unsigned)MAKO_ERI_REDUCED) return fail(MAKO_ERR_INVALID, "unknown flags");
     if (!basis || (nq > 0 && (!quartets || !out))) return fail(MAKO_ERR_INVALID, "NULL argument");
     if (nq < 0) return fail(MAKO_ERR_INVALID, "nq < 0");
     int dev = -1;
@@ -545,6 +608,8 @@ extern "C" mako_status mako_eri_batch(mako_basis basis, int nq, const int* quart
     PairSet set;
     mako_status st;
     if ((st = build_pair_set(basis, A, Bs, set, cuda_stream))) return st;
+    const bool lowp = (flags & MAKO_ERI_REDUCED) != 0;
+    if (lowp && (st = ensure_lowp(set, cuda_stream))) return st;
     cudaStream_t s = (cudaStream_t)cuda_stream;
     std::vector<std::unique_ptr<DevBuf>> keep;
     for (int X = 0; X < NBUCKET; ++X)
@@ -568,12 +633,23 @@ extern "C" mako_status mako_eri_batch(mako_basis basis, int nq, const int* quart
         a.out = out;
         a.boys = basis->d_boys.as<double>();
         a.diag = 0;
+        a.lowp = lowp ? 1 : 0;
         if ((st = launch_batch_class(X, Y, a, cuda_stream))) return st;
       }
     return cuda_check(cudaStreamSynchronize(s), "eri_batch sync");
   } catch (const std::exception& e) {
     return fail(MAKO_ERR_OOM, e.what());
   }
+}
+
+extern "C" mako_status mako_eri_batch(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,
+                                      void* cuda_stream) {
+  return eri_batch_impl(basis, nq, quartets, out, out_len, 0u, cuda_stream);
+}
+
+extern "C" mako_status mako_eri_batch_ex(mako_basis basis, int nq, const int* quartets, double* out, size_t out_len,
+                                         unsigned flags, void* cuda_stream) {
+  return eri_batch_impl(basis, nq, quartets, out, out_len, flags, cuda_stream);
 }
 
 extern "C" mako_status mako_boys(int n, const double* T, int mmax, double* out, void* cuda_stream) {

@@ -65,6 +65,16 @@ MK_HD constexpr int tpq_regs(int X, int Y) {
 MK_HD constexpr bool use_tpq(int X, int Y) { return Y <= 1 && tpq_regs(X, Y) <= 100; }
 MK_HD constexpr int class_kt(int X, int Y) { return use_tpq(X, Y) ? 32 : 16; }
 
+// reduced-precision tier: floats per primitive pair of the TF32 fragment-order copies of E~ (pairs.cu
+// build_lowp_kernel, read by eri_quant.cuh): GEMM1 A fragments (m16 x k8 tiles) and GEMM2 B fragments
+// (k8 x n8 tiles)
+MK_HD constexpr int lowp_a_floats(int la, int lb) {
+  return ((nsph(la) * nsph(lb) + 15) / 16) * ((nH(la + lb) + 7) / 8) * 128;
+}
+MK_HD constexpr int lowp_b_floats(int la, int lb) {
+  return ((nH(la + lb) + 7) / 8) * ((nsph(la) * nsph(lb) + 7) / 8) * 64;
+}
+
 // Pair buckets are ordered by (primitive-pair count group, Q descending): inside a group the
 // Schwarz-surviving kets of a bra are still a prefix, and the kets of one warp task share a similar
 // K_CD (uniform per-lane primitive loops).  Groups: K = 1, 2, 3, 4, 5-6, 7-9, 10-12, 13-16, 17-24,
@@ -124,6 +134,9 @@ struct PairView {
   const double* pdat;    // [nprim][4]: p, Px, Py, Pz
   const double* Ebra;    // [nprim][nab][nHab]  E~ with spherical transform, coefficients, 1/p folded
   const double* Eket;    // [nprim][nHab][nab]  (-1)^{|q|} E~^T
+  // reduced-precision tier (null until first requested): TF32 copies in mma fragment order
+  const float* EbraF;    // [nprim][MT16][KS8][32 lanes][4]  GEMM1 A fragments of E~
+  const float* EketF;    // [nprim][NT8(q)][NT8(cd)][32 lanes][2]  GEMM2 B fragments of (-1)^{|q|} E~^T
 };
 
 // arguments of a J/K class launch
@@ -152,6 +165,7 @@ struct JKArgs {
   double dw_thresh;
   const double* boys;               // Boys table
   int grid_div;                     // host side: grid = resident capacity / grid_div (concurrent classes)
+  int lowp;                         // host side: run the class's TF32-tier kernel (eri_quant.cuh)
 };
 
 // arguments of a store/diag class launch (eri_batch, Schwarz)
@@ -165,6 +179,7 @@ struct BatchArgs {
   double* out;
   const double* boys;
   int diag;               // 1 = Schwarz mode: out[qout[i]] = sqrt(max |(ab|ab)|)
+  int lowp;               // store mode: TF32-tier kernel where the class has one
 };
 
 }  // namespace mako

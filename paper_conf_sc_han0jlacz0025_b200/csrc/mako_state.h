@@ -45,6 +45,7 @@ struct PairBucket {
   std::vector<int> poff;           // [n+1]
   std::vector<int> seg;            // [NKGROUP+1] K-group segment starts (screened sets only)
   DevBuf d_shA, d_shB, d_Q, d_poff, d_pdat, d_Ebra, d_Eket;
+  DevBuf d_EbraF, d_EketF;         // TF32 fragment-order copies (reduced-precision tier, built on demand)
   int n() const { return (int)shA.size(); }
   PairView view() const;
 };
@@ -70,8 +71,10 @@ struct ClassPlan {
 
 struct Plan {
   double thresh = -1.0;
+  double tier = 0.0;               // > thresh: reduced-precision tier boundary (0 = FP64 only)
   int KT = 16;
-  std::vector<ClassPlan> cls;      // 55 classes
+  std::vector<ClassPlan> cls;      // 55 classes (FP64 tier)
+  std::vector<ClassPlan> cls_lo;   // 55 classes, TF32 tier (empty plans where the class has no TF32 kernel)
 };
 
 }  // namespace mako
@@ -116,9 +119,11 @@ void boys_table(std::vector<double>& tab);                                // com
 mako_status build_pair_set(const mako_basis_s* B, const std::vector<int> (&A)[NBUCKET],
                            const std::vector<int> (&Bsh)[NBUCKET], PairSet& out, void* stream);
 mako_status compute_schwarz(const mako_basis_s* B, PairSet& set, void* stream);
+mako_status ensure_lowp(PairSet& set, void* stream);   // TF32 operand copies of every bucket
 // class launches (eri_kernels*.cu)
 mako_status launch_jk_class(int X, int Y, const JKArgs& a, void* stream, int* nlaunch);
 mako_status launch_batch_class(int X, int Y, const BatchArgs& a, void* stream);
+bool class_has_lowp(int X, int Y);
 // class index (X >= Y) in 0..54
 inline int class_index(int X, int Y) { return X * (X + 1) / 2 + Y; }
 inline int bucket_la(int b) { int la = 0; while ((la + 1) * (la + 2) / 2 <= b) ++la; return la; }

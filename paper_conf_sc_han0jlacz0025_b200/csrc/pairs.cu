@@ -135,6 +135,8 @@ PairView PairBucket::view() const {
   v.pdat = d_pdat.as<double>();
   v.Ebra = d_Ebra.as<double>();
   v.Eket = d_Eket.as<double>();
+  v.EbraF = d_EbraF.as<float>();
+  v.EketF = d_EketF.as<float>();
   return v;
 }
 
@@ -189,6 +191,57 @@ mako_status build_pair_set(const mako_basis_s* B, const std::vector<int> (&A)[NB
     }
     // temporaries are freed at scope exit: make sure the kernel is done with them
     if ((st = cuda_check(cudaStreamSynchronize(s), "build_pair_set sync"))) return st;
+  }
+  return MAKO_OK;
+}
+
+// TF32 copies of E~ in mma.m16n8k8 fragment order (reduced-precision tier, eri_quant.cuh), zero
+// padded: A fragments of GEMM1 (lane (g,t): E~[16m+g][8k+t], E~[16m+g+8][8k+t], E~[16m+g][8k+t+4],
+// E~[16m+g+8][8k+t+4]) and B fragments of GEMM2 (lane (g,t): Ek[8n+2t][8j+g], Ek[8n+2t+1][8j+g],
+// Ek = (-1)^{|q|} E~^T).  One thread per output float.
+__global__ void build_lowp_kernel(int nab, int nh, long long total_a, long long total_b, const double* __restrict__ Ebra,
+                                  const double* __restrict__ Eket, float* __restrict__ EbraF,
+                                  float* __restrict__ EketF) {
+  const int MT = (nab + 15) / 16, KS = (nh + 7) / 8, NQ = (nh + 7) / 8, NC = (nab + 7) / 8;
+  const int AF = MT * KS * 128, BF = NQ * NC * 64;
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < total_a + total_b;
+       x += (long long)gridDim.x * blockDim.x) {
+    double v = 0.0;
+    if (x < total_a) {
+      const long long id = x / AF;
+      const int r = (int)(x % AF), mk = r / 128, lane = (r % 128) / 4, e = r % 4;
+      const int m = mk / KS, k = mk % KS, g = lane >> 2, t = lane & 3;
+      const int row = 16 * m + g + ((e & 1) ? 8 : 0), col = 8 * k + t + ((e & 2) ? 4 : 0);
+      if (row < nab && col < nh) v = Ebra[(size_t)id * nab * nh + (size_t)row * nh + col];
+      unsigned u;
+      asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(u) : "f"((float)v));
+      EbraF[x] = __uint_as_float(u);
+    } else {
+      const long long y = x - total_a, id = y / BF;
+      const int r = (int)(y % BF), nj = r / 64, lane = (r % 64) / 2, e = r % 2;
+      const int n = nj / NC, j = nj % NC, g = lane >> 2, t = lane & 3;
+      const int q = 8 * n + 2 * t + e, cd = 8 * j + g;
+      if (q < nh && cd < nab) v = Eket[(size_t)id * nab * nh + (size_t)q * nab + cd];
+      unsigned u;
+      asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(u) : "f"((float)v));
+      EketF[y] = __uint_as_float(u);
+    }
+  }
+}
+
+mako_status ensure_lowp(PairSet& set, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  for (int b = 0; b < NBUCKET; ++b) {
+    PairBucket& pb = set.b[b];
+    if (pb.d_EbraF.p) continue;
+    const long long np = std::max(pb.poff.empty() ? 0 : pb.poff.back(), 1);
+    const int nab = nsph(pb.la) * nsph(pb.lb), nh = nH(pb.la + pb.lb);
+    const long long ta = np * lowp_a_floats(pb.la, pb.lb), tb = np * lowp_b_floats(pb.la, pb.lb);
+    mako_status st;
+    if ((st = pb.d_EbraF.alloc(sizeof(float) * ta)) || (st = pb.d_EketF.alloc(sizeof(float) * tb))) return st;
+    build_lowp_kernel<<<1184, 256, 0, s>>>(nab, nh, ta, tb, pb.d_Ebra.as<double>(), pb.d_Eket.as<double>(),
+                                          pb.d_EbraF.as<float>(), pb.d_EketF.as<float>());
+    if ((st = cuda_check(cudaGetLastError(), "build_lowp_kernel"))) return st;
   }
   return MAKO_OK;
 }
@@ -289,7 +342,7 @@ extern "C" mako_status mako_shellpairs_screen(mako_basis basis, double thresh, v
       P->set.b[b].seg = seg[b];
       if ((st = upload_async(P->set.b[b].d_Q, Q2[b], s))) return st;
     }
-    if ((st = P->d_counters.alloc(sizeof(unsigned long long) * 64))) return st;
+    if ((st = P->d_counters.alloc(sizeof(unsigned long long) * 128))) return st;
     if ((st = cuda_check(cudaStreamSynchronize(s), "screen sync"))) return st;
     *out = P.release();
     return MAKO_OK;

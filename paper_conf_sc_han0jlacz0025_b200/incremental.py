@@ -13,7 +13,12 @@ full density (a) every `rebuild_every` builds, (b) when the threshold reaches ta
 converged Fock matrix then carries only tau_final-level screening error) and (c) when it has
 tightened by more than a factor `tighten` since the last full build.  The schedule (reading R18):
     tau_n = clip(tau_scale * max|Delta D_n|, tau_final, tau_loose)
-i.e. the neglected Fock contributions stay a fixed factor below the current density change.  All
+i.e. the neglected Fock contributions stay a fixed factor below the current density change.
+With `precision_scale` set, every build is also stage-aware mixed precision (mako_build_jk_mixed,
+SURVEY S8.f row 1; "relaxed precision thresholds during early iterations - favoring
+quantized kernels - and gradually tightening them as convergence nears"): quartets whose
+contribution bound Q_ab Q_cd max|D_build| is below thresh_fp64_n = precision_scale * max|Delta D_n|
+run the TF32 tier, so the reduced-precision share shrinks as the SCF converges (R21).  All
 device work runs in libmako's kernels; the Delta D / accumulation steps are torch tensor ops
 (plumbing).
 """
@@ -28,6 +33,14 @@ def tau_schedule(dmax, tau_final, tau_loose, tau_scale):
     return min(tau_loose, max(tau_final, t))
 
 
+def precision_schedule(dmax, precision_scale):
+    """thresh_fp64 of a build whose density change has max-norm `dmax` (None = FP64 only): quartets
+    whose contribution bound Q_ab Q_cd max|D_build| is below it run the TF32 tier (R21)."""
+    if precision_scale is None or not dmax > 0:
+        return None
+    return float(precision_scale) * float(dmax)
+
+
 class IncrementalJK:
     """Callable J/K builder for an SCF loop: ``J, K = inc(D)`` with D a device (or numpy) density.
 
@@ -35,13 +48,14 @@ class IncrementalJK:
     full or an incremental build, the threshold used, max|Delta D| and the device milliseconds."""
 
     def __init__(self, pairs, tau_final=None, tau_loose=1e-10, tau_scale=1e-7, rebuild_every=10, tighten=1e-3,
-                 device=None):
+                 device=None, precision_scale=None):
         self.pairs = pairs
         self.tau_final = float(pairs.tau if tau_final is None else tau_final)
         self.tau_loose = max(float(tau_loose), self.tau_final)
         self.tau_scale = float(tau_scale)
         self.rebuild_every = int(rebuild_every)
         self.tighten = float(tighten)
+        self.precision_scale = None if precision_scale is None else float(precision_scale)
         self.device = device or torch.device("cuda")
         self.D = self.J = self.K = None
         self.since_full = 0
@@ -64,20 +78,21 @@ class IncrementalJK:
         tau = tau_schedule(dmax, self.tau_final, self.tau_loose, self.tau_scale)
         full = (self.D is None or self.since_full >= self.rebuild_every or
                 (tau < self.tau_full and (tau <= self.tau_final or tau < self.tighten * self.tau_full)))
+        t64 = precision_schedule(dmax, self.precision_scale)
         if full:
-            J, K = build_jk(self.pairs, Dt, thresh=tau, density_screen=True)
+            J, K = build_jk(self.pairs, Dt, thresh=tau, density_screen=True, thresh_fp64=t64)
             self.J, self.K = J, K
             self.since_full = 0
             self.tau_full = tau
         else:
-            dJ, dK = build_jk(self.pairs, dD, thresh=tau, density_screen=True)
+            dJ, dK = build_jk(self.pairs, dD, thresh=tau, density_screen=True, thresh_fp64=t64)
             self.J = self.J + dJ
             self.K = self.K + dK
             self.since_full += 1
         self.D = Dt
         ev1.record()
         torch.cuda.synchronize()
-        self.history.append({"full": full, "tau": tau, "dmax": dmax, "ms": ev0.elapsed_time(ev1)})
+        self.history.append({"full": full, "tau": tau, "dmax": dmax, "thresh_fp64": t64, "ms": ev0.elapsed_time(ev1)})
         if numpy_in and return_numpy:
             return self.J.cpu().numpy(), self.K.cpu().numpy()
         return self.J, self.K

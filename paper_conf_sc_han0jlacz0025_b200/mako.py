@@ -131,11 +131,15 @@ class Pairs:
 
 
 MAKO_JK_DENSITY_SCREEN = 1
+MAKO_ERI_REDUCED = 1
 
 
-def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=None, density_screen=False):
+def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=None, density_screen=False,
+             thresh_fp64=None):
     """J_{mn} = sum (mn|ls) D_ls, K_{ml} = sum (mn|ls) D_ns on the GPU (north_star).  Async on `stream`
-    (density_screen=True: mako_build_jk_ex with MAKO_JK_DENSITY_SCREEN, which synchronises `stream`)."""
+    (density_screen=True: mako_build_jk_ex with MAKO_JK_DENSITY_SCREEN, which synchronises `stream`).
+    thresh_fp64: stage-aware reduced-precision build (mako_build_jk_mixed; synchronises `stream`):
+    quartets whose contribution bound Q_ab Q_cd max|D| is below ~thresh_fp64 run the TF32 tier."""
     n = pairs.basis.nbf
     if D.shape != (n, n):
         raise ValueError(f"D must be {n}x{n}")
@@ -144,7 +148,11 @@ def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=N
     if K is None:
         K = torch.empty_like(D)
     t = float(pairs.tau if thresh is None else thresh)
-    if density_screen:
+    if thresh_fp64 is not None:
+        check(pairs._lib.mako_build_jk_mixed(pairs.handle, _dev_ptr(D, "D"), t, float(thresh_fp64),
+                                             MAKO_JK_DENSITY_SCREEN if density_screen else 0, _dev_ptr(J, "J"),
+                                             _dev_ptr(K, "K"), int(shard), int(nshards), _stream_ptr(stream)))
+    elif density_screen:
         check(pairs._lib.mako_build_jk_ex(pairs.handle, _dev_ptr(D, "D"), t, MAKO_JK_DENSITY_SCREEN, _dev_ptr(J, "J"),
                                           _dev_ptr(K, "K"), int(shard), int(nshards), _stream_ptr(stream)))
     else:
@@ -153,14 +161,23 @@ def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=N
     return J, K
 
 
-def eri_batch(basis, quartets, stream=None, device=None):
-    """Shell-quartet ERI blocks (test entry).  Returns a list of numpy-shaped torch tensors on the GPU."""
+def class_reduced():
+    """[55] bool: classes with a reduced-precision (TF32) kernel (mako_class_reduced)."""
+    m = np.zeros(_lib.NCLASS, np.int32)
+    check(_lib.load().mako_class_reduced(m.ctypes.data_as(ctypes.POINTER(ctypes.c_int))))
+    return m.astype(bool)
+
+
+def eri_batch(basis, quartets, stream=None, device=None, reduced=False):
+    """Shell-quartet ERI blocks (test entry).  Returns a list of numpy-shaped torch tensors on the GPU.
+    reduced=True: mako_eri_batch_ex with MAKO_ERI_REDUCED (the TF32 tier where the class has one)."""
     q, qp = _i32(np.asarray(quartets).reshape(-1, 4))
     # out-of-range shells are left to the C ABI to reject (MAKO_ERR_INVALID)
     nf = lambda s: 2 * int(basis.l[s]) + 1 if 0 <= s < basis.nshell else 0
     sizes = [int(np.prod([nf(s) for s in row])) for row in q]
     out = torch.empty(sum(sizes), dtype=torch.float64, device=device or "cuda")
-    check(basis._lib.mako_eri_batch(basis.handle, len(q), qp, _dev_ptr(out, "out"), out.numel(), _stream_ptr(stream)))
+    check(basis._lib.mako_eri_batch_ex(basis.handle, len(q), qp, _dev_ptr(out, "out"), out.numel(),
+                                       MAKO_ERI_REDUCED if reduced else 0, _stream_ptr(stream)))
     res, o = [], 0
     for row, s in zip(q, sizes):
         res.append(out[o:o + s].view(*[2 * basis.l[x] + 1 for x in row]))

@@ -62,3 +62,23 @@ def test_errors_without_gpu():
     st = lib.mako_basis_create(2, ip(Z), dp(xyz), 2, ip(at), ip(l), ip(npr), dp(e), dp(c), 0, ctypes.byref(h))
     assert st == 2
     assert lib.mako_build_jk(None, None, 0.0, None, None, 0, 1, None) == 1
+
+
+def test_reduced_precision_tier_boundary():
+    """the TF32 tier exists in the library (SASS HMMA.1688.F32.TF32 next to DMMA), covers
+    every high-l class (L >= 8, where the basis transformation dominates), and the mixed build
+    validates its arguments before touching the device."""
+    import subprocess
+    from paper_conf_sc_han0jlacz0025_b200 import _lib, class_reduced
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", _lib.LIB_PATH], capture_output=True, text=True).stdout
+    assert "HMMA.1688.F32.TF32" in sass
+    m = class_reduced()
+    bl = [(0, 0), (1, 0), (1, 1), (2, 0), (2, 1), (2, 2), (3, 0), (3, 1), (3, 2), (3, 3)]
+    for X in range(10):
+        for Y in range(X + 1):
+            if sum(bl[X]) + sum(bl[Y]) >= 8:
+                assert m[X * (X + 1) // 2 + Y], (bl[X], bl[Y])
+    assert not m[0] and not m[1]  # (ss|ss), (ps|ss): lane-per-ket FP64 only
+    lib = _lib.load()
+    assert lib.mako_build_jk_mixed(None, None, 0.0, 1e-6, 0, None, None, 0, 1, None) == 1
+    assert lib.mako_class_reduced(None) == 1
