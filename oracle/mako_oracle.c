@@ -239,24 +239,30 @@ int orc_nbf(int nshell, const int* l, int pure) {
 /* in:  [gidx(e) for |e| <= la+lb][nf]  (only |e| >= la used)              */
 /* out: [ncart(la)][ncart(lb)][nf]                                         */
 /* ------------------------------------------------------------------ */
-static void hrr(int la, int lb, const double AB[3], int nf, const double* in, double* out) {
+/* The ERI pipeline (VRR, HRR, contraction, spherical transform) runs in long double: the HRR's
+ * cancellation at l = 4 with diffuse exponents costs ~1e-10 absolute in double (measured as the
+ * spread between permuted evaluations of one quartet), the size of the north_star ERI bar
+ * (reading R22). */
+typedef long double real_t;
+
+static void hrr(int la, int lb, const real_t AB[3], int nf, const real_t* in, real_t* out) {
   int Lab = la + lb;
   if (lb == 0) {
     int xyz[3 * 15 * 2];
     cart_list(la, xyz);
     for (int i = 0; i < ncart(la); ++i)
       memcpy(out + (size_t)i * nf, in + (size_t)gidx(xyz[3 * i], xyz[3 * i + 1], xyz[3 * i + 2]) * nf,
-             sizeof(double) * nf);
+             sizeof(real_t) * nf);
     return;
   }
   /* T_j[e][b] for |b| = j, |e| in [la, Lab - j]; stored as [gidx(e)][cidx(b)][nf] */
   int ne = ncum(Lab);
-  double* prev = (double*)calloc((size_t)ne * 1 * nf, sizeof(double));
-  memcpy(prev, in, sizeof(double) * (size_t)ne * nf);
+  real_t* prev = (real_t*)calloc((size_t)ne * 1 * nf, sizeof(real_t));
+  memcpy(prev, in, sizeof(real_t) * (size_t)ne * nf);
   int nbprev = 1;
   for (int j = 1; j <= lb; ++j) {
     int nb = ncart(j);
-    double* cur = (double*)calloc((size_t)ne * nb * nf, sizeof(double));
+    real_t* cur = (real_t*)calloc((size_t)ne * nb * nf, sizeof(real_t));
     int bl[3 * 45];
     cart_list(j, bl);
     for (int le = la; le <= Lab - j; ++le) {
@@ -271,9 +277,9 @@ static void hrr(int la, int lb, const double AB[3], int nf, const double* in, do
           bm[d] -= 1;
           int ep[3] = {ex, ey, ez};
           ep[d] += 1;
-          const double* t1 = prev + ((size_t)gidx(ep[0], ep[1], ep[2]) * nbprev + cidx(bm[0], bm[1], bm[2])) * nf;
-          const double* t2 = prev + ((size_t)gidx(ex, ey, ez) * nbprev + cidx(bm[0], bm[1], bm[2])) * nf;
-          double* o = cur + ((size_t)gidx(ex, ey, ez) * nb + ib) * nf;
+          const real_t* t1 = prev + ((size_t)gidx(ep[0], ep[1], ep[2]) * nbprev + cidx(bm[0], bm[1], bm[2])) * nf;
+          const real_t* t2 = prev + ((size_t)gidx(ex, ey, ez) * nbprev + cidx(bm[0], bm[1], bm[2])) * nf;
+          real_t* o = cur + ((size_t)gidx(ex, ey, ez) * nb + ib) * nf;
           for (int k = 0; k < nf; ++k) o[k] = t1[k] + AB[d] * t2[k];
         }
       }
@@ -288,21 +294,21 @@ static void hrr(int la, int lb, const double AB[3], int nf, const double* in, do
     for (int ib = 0; ib < ncart(lb); ++ib)
       memcpy(out + ((size_t)ia * ncart(lb) + ib) * nf,
              prev + ((size_t)gidx(al[3 * ia], al[3 * ia + 1], al[3 * ia + 2]) * nbprev + ib) * nf,
-             sizeof(double) * nf);
+             sizeof(real_t) * nf);
   free(prev);
 }
 
 /* ------------------------------------------------------------------ */
 /* Obara-Saika VRR for one primitive quartet, accumulated (x coef) into   */
 /* acc[gidx(e)][gidx(f)] for |e| <= Le, |f| <= Lf  (only m = 0 kept).        */
-/* work: (ncum(Le) * ncum(Lf) * (Le+Lf+1)) doubles                          */
+/* work: (ncum(Le) * ncum(Lf) * (Le+Lf+1)) real_ts                          */
 /* ------------------------------------------------------------------ */
-static void os_vrr_prim(int Le, int Lf, double a, const double* A, double b, const double* B, double c,
-                        const double* C, double d, const double* D, double coef, double* acc, double* work) {
+static void os_vrr_prim(int Le, int Lf, real_t a, const double* A, real_t b, const double* B, real_t c,
+                        const double* C, real_t d, const double* D, real_t coef, real_t* acc, real_t* work) {
   const int L = Le + Lf;
   const int nE = ncum(Le), nF = ncum(Lf), nM = L + 1;
-  double p = a + b, q = c + d, rho = p * q / (p + q);
-  double P[3], Q[3], W[3], PA[3], QC[3], WP[3], WQ[3], AB2 = 0, CD2 = 0, PQ2 = 0;
+  real_t p = a + b, q = c + d, rho = p * q / (p + q);
+  real_t P[3], Q[3], W[3], PA[3], QC[3], WP[3], WQ[3], AB2 = 0, CD2 = 0, PQ2 = 0;
   for (int i = 0; i < 3; ++i) {
     P[i] = (a * A[i] + b * B[i]) / p;
     Q[i] = (c * C[i] + d * D[i]) / q;
@@ -314,9 +320,10 @@ static void os_vrr_prim(int Le, int Lf, double a, const double* A, double b, con
   }
   long double F[ORC_LTOT + 1];
   boys_ld(L, (long double)(rho * PQ2), F);
-  double pref = 2.0 * pow(M_PI, 2.5) / (p * q * sqrt(p + q)) * exp(-a * b / p * AB2 - c * d / q * CD2);
+  real_t pref = 2.0L * powl(3.14159265358979323846264338327950288L, 2.5L) / (p * q * sqrtl(p + q)) *
+                expl(-a * b / p * AB2 - c * d / q * CD2);
 #define V(ei, fi, m) work[((size_t)(ei) * nF + (fi)) * nM + (m)]
-  for (int m = 0; m <= L; ++m) V(0, 0, m) = pref * (double)F[m];
+  for (int m = 0; m <= L; ++m) V(0, 0, m) = pref * F[m];
   /* build e (f = 0) */
   for (int le = 1; le <= Le; ++le) {
     int el[3 * 91];
@@ -330,7 +337,7 @@ static void os_vrr_prim(int Le, int Lf, double a, const double* A, double b, con
       int g2 = -1;
       if (n1 > 0) { int e2[3] = {e1[0], e1[1], e1[2]}; e2[i] -= 1; g2 = gidx(e2[0], e2[1], e2[2]); }
       for (int m = 0; m <= L - le; ++m) {
-        double v = PA[i] * V(g1, 0, m) + WP[i] * V(g1, 0, m + 1);
+        real_t v = PA[i] * V(g1, 0, m) + WP[i] * V(g1, 0, m + 1);
         if (n1 > 0) v += n1 / (2.0 * p) * (V(g2, 0, m) - rho / p * V(g2, 0, m + 1));
         V(g, 0, m) = v;
       }
@@ -357,7 +364,7 @@ static void os_vrr_prim(int Le, int Lf, double a, const double* A, double b, con
           int ge = -1;
           if (e[i] > 0) { int em[3] = {e[0], e[1], e[2]}; em[i] -= 1; ge = gidx(em[0], em[1], em[2]); }
           for (int m = 0; m <= L - le - lf; ++m) {
-            double v = QC[i] * V(g, h1, m) + WQ[i] * V(g, h1, m + 1);
+            real_t v = QC[i] * V(g, h1, m) + WQ[i] * V(g, h1, m + 1);
             if (n1 > 0) v += n1 / (2.0 * q) * (V(g, h2, m) - rho / q * V(g, h2, m + 1));
             if (e[i] > 0) v += e[i] / (2.0 * (p + q)) * V(ge, h1, m + 1);
             V(g, h, m) = v;
@@ -377,65 +384,65 @@ static void eri_block(const basis_t* B, int sa, int sb, int sc, int sd, double* 
   int Le = la + lb, Lf = lc + ld;
   int nE = ncum(Le), nF = ncum(Lf);
   const double *A = B->xyz + 3 * sa, *Bc = B->xyz + 3 * sb, *C = B->xyz + 3 * sc, *D = B->xyz + 3 * sd;
-  double* acc = (double*)calloc((size_t)nE * nF, sizeof(double));
-  double* work = (double*)malloc(sizeof(double) * (size_t)nE * nF * (Le + Lf + 1));
+  real_t* acc = (real_t*)calloc((size_t)nE * nF, sizeof(real_t));
+  real_t* work = (real_t*)malloc(sizeof(real_t) * (size_t)nE * nF * (Le + Lf + 1));
   for (int i = 0; i < B->nprim[sa]; ++i)
     for (int j = 0; j < B->nprim[sb]; ++j)
       for (int k = 0; k < B->nprim[sc]; ++k)
         for (int m = 0; m < B->nprim[sd]; ++m) {
           int pi = B->poff[sa] + i, pj = B->poff[sb] + j, pk = B->poff[sc] + k, pm = B->poff[sd] + m;
-          double coef = B->cn[pi] * B->cn[pj] * B->cn[pk] * B->cn[pm];
+          real_t coef = (real_t)B->cn[pi] * B->cn[pj] * B->cn[pk] * B->cn[pm];
           os_vrr_prim(Le, Lf, B->exps[pi], A, B->exps[pj], Bc, B->exps[pk], C, B->exps[pm], D, coef, acc, work);
         }
   free(work);
   /* bra HRR: [e][f] -> [a][b][f] */
-  double AB[3] = {A[0] - Bc[0], A[1] - Bc[1], A[2] - Bc[2]};
-  double CD[3] = {C[0] - D[0], C[1] - D[1], C[2] - D[2]};
+  real_t AB[3] = {A[0] - Bc[0], A[1] - Bc[1], A[2] - Bc[2]};
+  real_t CD[3] = {C[0] - D[0], C[1] - D[1], C[2] - D[2]};
   int nca = ncart(la), ncb = ncart(lb), ncc = ncart(lc), ncd = ncart(ld);
-  double* t1 = (double*)malloc(sizeof(double) * (size_t)nca * ncb * nF);
+  real_t* t1 = (real_t*)malloc(sizeof(real_t) * (size_t)nca * ncb * nF);
   hrr(la, lb, AB, nF, acc, t1);
   /* transpose to [f][ab] for the ket HRR */
   int nab = nca * ncb;
-  double* t2 = (double*)malloc(sizeof(double) * (size_t)nF * nab);
+  real_t* t2 = (real_t*)malloc(sizeof(real_t) * (size_t)nF * nab);
   for (int x = 0; x < nab; ++x)
     for (int h = 0; h < nF; ++h) t2[(size_t)h * nab + x] = t1[(size_t)x * nF + h];
-  double* t3 = (double*)malloc(sizeof(double) * (size_t)ncc * ncd * nab);
+  real_t* t3 = (real_t*)malloc(sizeof(real_t) * (size_t)ncc * ncd * nab);
   hrr(lc, ld, CD, nab, t2, t3);
   /* cart[a][b][c][d] */
-  double* cart = (double*)malloc(sizeof(double) * (size_t)nab * ncc * ncd);
+  real_t* cart = (real_t*)malloc(sizeof(real_t) * (size_t)nab * ncc * ncd);
   for (int x = 0; x < nab; ++x)
     for (int y = 0; y < ncc * ncd; ++y) cart[(size_t)x * ncc * ncd + y] = t3[(size_t)y * nab + x];
   free(acc); free(t1); free(t2); free(t3);
   if (!B->pure) {
-    memcpy(out, cart, sizeof(double) * (size_t)nab * ncc * ncd);
+    for (size_t x = 0; x < (size_t)nab * ncc * ncd; ++x) out[x] = (double)cart[x];
     free(cart);
     return;
   }
   /* spherical transform index by index */
   int ls[4] = {la, lb, lc, ld};
   int nin[4] = {nca, ncb, ncc, ncd};
-  double* cur = cart;
+  real_t* cur = cart;
   int dims[4] = {nca, ncb, ncc, ncd};
   for (int ax = 0; ax < 4; ++ax) {
     int no = nsph(ls[ax]);
     int pre = 1, post = 1;
     for (int k = 0; k < ax; ++k) pre *= dims[k];
     for (int k = ax + 1; k < 4; ++k) post *= dims[k];
-    double* nxt = (double*)calloc((size_t)pre * no * post, sizeof(double));
+    real_t* nxt = (real_t*)calloc((size_t)pre * no * post, sizeof(real_t));
     for (int x = 0; x < pre; ++x)
       for (int o = 0; o < no; ++o)
         for (int i = 0; i < nin[ax]; ++i) {
-          double cf = sph_tab[ls[ax]][o][i];
+          real_t cf = sph_tab[ls[ax]][o][i];
           if (cf == 0.0) continue;
-          const double* src = cur + ((size_t)x * nin[ax] + i) * post;
-          double* dst = nxt + ((size_t)x * no + o) * post;
+          const real_t* src = cur + ((size_t)x * nin[ax] + i) * post;
+          real_t* dst = nxt + ((size_t)x * no + o) * post;
           for (int y = 0; y < post; ++y) dst[y] += cf * src[y];
         }
     free(cur);
     cur = nxt;
     dims[ax] = no;
   }
-  memcpy(out, cur, sizeof(double) * (size_t)dims[0] * dims[1] * dims[2] * dims[3]);
+  for (size_t x = 0; x < (size_t)dims[0] * dims[1] * dims[2] * dims[3]; ++x) out[x] = (double)cur[x];
   free(cur);
 }
 
@@ -827,10 +834,13 @@ int orc_one_electron(BASIS_ARGS, int natm, const double* Z, const double* axyz, 
             }
           prim_V_acc(la, lb, exps[pi], A, exps[pj], Bc, natm, Z, axyz, cf, vacc);
         }
-      double ABv[3] = {A[0] - Bc[0], A[1] - Bc[1], A[2] - Bc[2]};
-      hrr(la, lb, ABv, 1, vacc, vab);
-      for (int x = 0; x < nca * ncb; ++x) cv[x] = vab[x];
-      free(vacc); free(vab);
+      real_t ABv[3] = {A[0] - Bc[0], A[1] - Bc[1], A[2] - Bc[2]};
+      real_t* vaccl = (real_t*)malloc(sizeof(real_t) * ncum(la + lb));
+      real_t* vabl = (real_t*)malloc(sizeof(real_t) * nca * ncb);
+      for (int x = 0; x < ncum(la + lb); ++x) vaccl[x] = vacc[x];
+      hrr(la, lb, ABv, 1, vaccl, vabl);
+      for (int x = 0; x < nca * ncb; ++x) cv[x] = (double)vabl[x];
+      free(vacc); free(vab); free(vaccl); free(vabl);
       double os[225], ot[225], ov[225];
       sph_2idx(&B, la, lb, cs, os);
       sph_2idx(&B, la, lb, ct, ot);

@@ -45,7 +45,7 @@ def norm2_mp(alpha, powers):
 def cart_eri_mp(exps, centers, powers):
     """Primitive Cartesian ERI via center derivatives of the closed-form (ss|ss):
     u^1 g = D g/(2a), u^2 g = D^2 g/(4a^2) + g/(2a), u^3 g = D^3 g/(8a^3) + 3 D g/(4a^2),
-    D = d/dA_x acting on exp(-a (x-A_x)^2)."""
+    u^4 g = D^4 g/(16a^4) + 3 D^2 g/(4a^3) + 3 g/(4a^2),  D = d/dA_x acting on exp(-a (x-A_x)^2)."""
     a = [mp.mpf(e) for e in exps]
     X0 = [mp.mpf(v) for c in centers for v in c]
 
@@ -59,6 +59,8 @@ def cart_eri_mp(exps, centers, powers):
             return [(2, 1 / (4 * al ** 2)), (0, 1 / (2 * al))]
         if n == 3:
             return [(3, 1 / (8 * al ** 3)), (1, 3 / (4 * al ** 2))]
+        if n == 4:  # D^4 g = 16a^4 u^4 g - 48a^3 u^2 g + 12a^2 g
+            return [(4, 1 / (16 * al ** 4)), (2, 3 / (4 * al ** 3)), (0, 3 / (4 * al ** 2))]
         raise ValueError
 
     terms = [((), mp.mpf(1))]
@@ -126,6 +128,13 @@ CASES = [
     ((0, 0, 3, 2), (1.0, 0.6, 0.9, 1.4),
      ((0.0, 0.0, 0.3), (0.7, 0.1, -0.2), (-0.3, 0.5, 0.4), (0.5, -0.6, 0.9)),
      ((0, 0, 0), (0, 0, 0), (0, 0, 3), (1, 0, 1))),
+    # g functions (row f3): (g_xxyz s | p_x s) and (s s | g_zzzz s)
+    ((4, 0, 1, 0), (0.9, 1.3, 0.7, 0.6),
+     ((0.1, -0.2, 0.3), (-0.7, 0.4, 0.2), (0.5, 0.6, -0.4), (0.3, -0.5, 0.8)),
+     ((2, 1, 1), (0, 0, 0), (1, 0, 0), (0, 0, 0))),
+    ((0, 0, 4, 0), (1.1, 0.8, 0.6, 1.5),
+     ((0.0, 0.2, -0.1), (0.6, -0.3, 0.4), (-0.4, 0.1, 0.7), (0.2, 0.9, -0.5)),
+     ((0, 0, 0), (0, 0, 0), (0, 0, 4), (0, 0, 0))),
 ]
 
 
