@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """bench.py -- BASELINE.json metric "Fock J+K build s/iter & ERI contraction TFLOP/s at 1/2/4/8 B200".
 
-A step = one direct-SCF J/K build (mako_build_jk: all 55 angular-momentum classes -- Boys, R
+A step = one direct-SCF J/K build (mako_build_jk: all angular-momentum classes (55 for the l <= 3 bases benched) -- Boys, R
 recursion, the two DMMA Hermite->AO contractions, FP64 digestion -- plus, for N > 1, broadcast(D)
 and all_reduce(J, K)) over the valinomycin-sized def2-TZVP workload (BASELINE.json configs[3],
 "J/K build at 1/2/4/8 GPUs"; configs[4] is an 8-GPU-only config and configs[0..2] are parity cases).
@@ -79,7 +79,7 @@ def workload_flops(sh, Q, tau, prim_eps=PRIM_EPS):
         v = sorted([x for x in buckets[k] if x[0] * qmax >= tau], key=lambda x: (kgroup(x[1]), -x[0]))
         buckets[k] = (np.array([x[0] for x in v]), np.array([x[1] for x in v], np.int64),
                       np.array([kgroup(x[1]) for x in v], np.int64))
-    bl = lambda b: [(0, 0), (1, 0), (1, 1), (2, 0), (2, 1), (2, 2), (3, 0), (3, 1), (3, 2), (3, 3)][b]
+    bl = lambda b: [(la, lb) for la in range(5) for lb in range(la + 1)][b]
     total, nq = 0.0, 0
     for X in buckets:
         for Y in buckets:
@@ -298,7 +298,7 @@ def run_mako(args):
     # stage-aware reduced-precision tier (mako_build_jk_mixed): same workload, quartets
     # with Q_ab Q_cd max|D| < thresh_fp64 in the TF32 tier; error of the two-electron energy vs FP64
     mixed = None
-    names_ = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff"]
+    names_ = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff", "gs", "gp", "gd", "gf", "gg"]
     if args.mixed > 0 and world == 1:
         Jm, Km = torch.empty_like(D), torch.empty_like(D)
         build_jk(P, D, J=Jm, K=Km, stream=stream, thresh_fp64=args.mixed)
@@ -361,7 +361,7 @@ def run_mako(args):
     c = int(np.argmax(cls_ms))
     per_launch_ms = cls_ms[c] / max(cls_n[c], 1)
     achieved = cls_flops[c] / (per_launch_ms * 1e-3) / 1e12
-    names = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff"]
+    names = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff", "gs", "gp", "gd", "gf", "gg"]
     X = int((math.isqrt(8 * c + 1) - 1) // 2)
     Y = c - X * (X + 1) // 2
     traffic = None

@@ -48,7 +48,7 @@
 extern "C" {
 #endif
 
-#define MAKO_LMAX 3
+#define MAKO_LMAX 4
 
 typedef enum {
   MAKO_OK = 0,
@@ -153,9 +153,9 @@ mako_status mako_class_reduced(int* mask);
 /* Number of CUDA kernels one mako_build_jk call launches for these arguments (for bench accounting). */
 mako_status mako_build_jk_launches(mako_pairs pairs, double thresh, int shard, int nshards, int* n_launches);
 
-/* Number of angular-momentum classes (bra bucket X >= ket bucket Y over the 10 (la>=lb) pair
- * buckets ss ps pp ds dp dd fs fp fd ff): class index c = X(X+1)/2 + Y. */
-#define MAKO_NCLASS 55
+/* Number of angular-momentum classes (bra bucket X >= ket bucket Y over the 15 (la>=lb) pair
+ * buckets ss ps pp ds dp dd fs fp fd ff gs gp gd gf gg): class index c = X(X+1)/2 + Y. */
+#define MAKO_NCLASS 120
 
 /* Per-class algorithmic GEMM FLOPs (same definition as mako_pairs_flops) and quartet counts of
  * shard `shard`/`nshards` at thresh.  flops, quartets, prim_quartets: HOST arrays of MAKO_NCLASS (any NULL). */

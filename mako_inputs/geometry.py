@@ -143,6 +143,9 @@ CONFIGS = {
     "gly10-ccpvtz": (lambda: glycine_oligomer(10), "cc-pvtz"),
     # not a BASELINE config: the SCF-timing case of the incremental builder
     "gly10-def2svp": (lambda: glycine_oligomer(10), "def2-svp"),
+    # not BASELINE configs: g functions (cc-pVQZ family of PAPER.md:L392)
+    "h2o-ccpvqz": (h2o_baseline, "cc-pvqz"),
+    "benzene-ccpvqz": (benzene, "cc-pvqz"),
     "valinomycin-def2tzvp": (lambda: random_packed(VALINOMYCIN, name="valinomycin-sized"), "def2-tzvp"),
     "ubiquitin-def2tzvp": (lambda: random_packed(UBIQUITIN, name="ubiquitin-sized"), "def2-tzvp"),
 }

@@ -13,7 +13,7 @@ if os.environ.get("MAKO_LIB"):
     LIB_PATH = os.path.join(HERE, "libmako_%s.so" % os.environ["MAKO_LIB"])
 
 MAKO_OK = 0
-NCLASS = 55
+NCLASS = 120  # MAKO_NCLASS (l <= 4: 15 pair buckets)
 STATUS = {0: "MAKO_OK", 1: "MAKO_ERR_INVALID", 2: "MAKO_ERR_UNSUPPORTED", 3: "MAKO_ERR_CUDA", 4: "MAKO_ERR_OOM",
           5: "MAKO_ERR_STATE"}
 

@@ -24,7 +24,7 @@ constexpr double TWO_PI_52 = 34.98683665524972497;  // 2 pi^{5/2}
 constexpr double PI_D = 3.14159265358979323846;
 
 MK_HD constexpr int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
-MK_HD constexpr int bla(int b) { return b >= 6 ? 3 : (b >= 3 ? 2 : (b >= 1 ? 1 : 0)); }
+MK_HD constexpr int bla(int b) { return b_la(b); }
 MK_HD constexpr int blb(int b) { return b - bla(b) * (bla(b) + 1) / 2; }
 
 template <int LA_, int LB_, int LC_, int LD_>

@@ -44,9 +44,20 @@ constexpr bool has_lowp() {
   return !use_tpq(X, Y) && !use_kf<X, Y>() && !use_kf_swap<X, Y>() && !use_slab<X, Y>();
 }
 
+// warps per CTA of the warp-per-quartet kernels: 4, fewer when the per-warp SMEM of a class does
+// not fit (l = 4 classes: (gg|gg) runs 2 warps per CTA)
+constexpr size_t SMEM_CTA_MAX = 227 * 1024 - 1024;
+template <class C, int WD>
+__host__ __device__ constexpr int warps_for() {
+  constexpr size_t w = (SMEM_CTA_MAX - C::HTAB_BYTES - C::RTAB_BYTES) / (sizeof(double) * WD);
+  static_assert(w >= 1, "class does not fit in shared memory");
+  return w >= CTA_WARPS ? CTA_WARPS : (int)w;
+}
+template <class C>
+__host__ __device__ constexpr int jk_warps() { return warps_for<C, C::WARP_DBL>(); }
 template <class C>
 __host__ __device__ constexpr size_t cta_smem_bytes() {
-  return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)CTA_WARPS * C::WARP_DBL;
+  return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)jk_warps<C>() * C::WARP_DBL;
 }
 
 // occupancy cap (4 CTAs/SM, <= 128 registers) measured faster for the fd-bra classes and (fp|dd) only
@@ -147,8 +158,10 @@ __device__ void store_block(const BatchArgs& a, int qi, const double* __restrict
 // Reduced-precision tier of the persistent J/K kernel (eri_quant.cuh): the task loop and the FP64
 // digestion of jk_body, the TF32 basis transformation of quartet_block_q.
 template <class C>
+__host__ __device__ constexpr int q_warps() { return warps_for<C, ClsQ<C>::WARP_DBL>(); }
+template <class C>
 __host__ __device__ constexpr size_t cta_smem_bytes_q() {
-  return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)CTA_WARPS * ClsQ<C>::WARP_DBL;
+  return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)q_warps<C>() * ClsQ<C>::WARP_DBL;
 }
 template <int X, int Y, bool DW = false>
 __global__ void __launch_bounds__(CTA_THREADS) jk_kernel_q(JKArgs a) {
@@ -220,7 +233,7 @@ __global__ void __launch_bounds__(CTA_THREADS) batch_kernel_q(BatchArgs a) {
   double* Rbuf = wbase + (size_t)warp * Q::WARP_DBL;
   double* V = Rbuf + C::W_R;
   float* R32 = reinterpret_cast<float*>(Rbuf + C::WARP_DBL);
-  for (int qi = blockIdx.x * CTA_WARPS + warp; qi < a.nq; qi += gridDim.x * CTA_WARPS) {
+  for (int qi = blockIdx.x * (blockDim.x >> 5) + warp; qi < a.nq; qi += gridDim.x * (blockDim.x >> 5)) {
     quartet_block_q<C>(a.bra, a.qbra[qi], a.ket, a.qket[qi], Rbuf, R32, V, htab, rtab, a.boys, lane);
     store_block<C>(a, qi, V, lane);
     __syncwarp();
@@ -240,7 +253,7 @@ __global__ void __launch_bounds__(CTA_THREADS) batch_kernel(BatchArgs a) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   double* Rbuf = wbase + (size_t)warp * C::WARP_DBL;
   double* V = Rbuf + C::W_R;
-  for (int qi = blockIdx.x * CTA_WARPS + warp; qi < a.nq; qi += gridDim.x * CTA_WARPS) {
+  for (int qi = blockIdx.x * (blockDim.x >> 5) + warp; qi < a.nq; qi += gridDim.x * (blockDim.x >> 5)) {
     const int P = a.qbra[qi], R = a.qket[qi];
     quartet_block<C>(a.bra, P, a.ket, R, Rbuf, V, htab, rtab, a.boys, lane);
     if (a.diag) {
@@ -286,7 +299,7 @@ int jk_blocks_per_sm() {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, slab_jk_kernel<X, Y>, CTA_THREADS, ss);
     } else {
       if (set_smem_attr<X, Y>((const void*)jk_kernel_ptr<X, Y>(), smem)) return 1;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel_ptr<X, Y>(), CTA_THREADS, smem);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel_ptr<X, Y>(), 32 * jk_warps<C>(), smem);
     }
     cached = nb < 1 ? 1 : nb;
   }
@@ -303,7 +316,9 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   const int bps = jk_blocks_per_sm<X, Y>();
-  long long want = (ntask + CTA_WARPS - 1) / CTA_WARPS;
+  constexpr int WPC = (use_kf_swap<X, Y>() || use_kf<X, Y>() || use_tpq(X, Y) || use_slab<X, Y>()) ? CTA_WARPS
+                                                                                                 : jk_warps<C>();
+  long long want = (ntask + WPC - 1) / WPC;
   long long cap = (long long)nsm * bps / (a.grid_div > 1 ? a.grid_div : 1);
   if (cap < nsm) cap = nsm;
   const int grid = (int)(want < cap ? want : cap);
@@ -319,12 +334,13 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
         if (set_smem_attr<X, Y>((const void*)jk_kernel_q<X, Y>, sq) ||
             set_smem_attr<X, Y>((const void*)jk_kernel_q<X, Y, true>, sq))
           return MAKO_ERR_CUDA;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bq, jk_kernel_q<X, Y>, CTA_THREADS, sq);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bq, jk_kernel_q<X, Y>, 32 * q_warps<C>(), sq);
         if (bq < 1) bq = 1;
       }
-      const long long gq = std::min<long long>(want, std::max<long long>((long long)nsm * bq, nsm));
-      if (a.dsh) jk_kernel_q<X, Y, true><<<(int)gq, CTA_THREADS, sq, cs>>>(a);
-      else jk_kernel_q<X, Y><<<(int)gq, CTA_THREADS, sq, cs>>>(a);
+      constexpr int QW = q_warps<C>();
+      const long long gq = std::min<long long>((ntask + QW - 1) / QW, std::max<long long>((long long)nsm * bq, nsm));
+      if (a.dsh) jk_kernel_q<X, Y, true><<<(int)gq, 32 * QW, sq, cs>>>(a);
+      else jk_kernel_q<X, Y><<<(int)gq, 32 * QW, sq, cs>>>(a);
       cudaError_t e = cudaGetLastError();
       if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("jk_kernel_q launch: ") + cudaGetErrorString(e));
       if (nlaunch) ++*nlaunch;
@@ -358,9 +374,9 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   } else {
     if (a.dsh) {
       if (set_smem_attr<X, Y>((const void*)jk_kernel_ptr<X, Y, true>(), smem)) return MAKO_ERR_CUDA;
-      jk_kernel_ptr<X, Y, true>()<<<grid, CTA_THREADS, smem, cs>>>(a);
+      jk_kernel_ptr<X, Y, true>()<<<grid, 32 * WPC, smem, cs>>>(a);
     } else {
-      jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, smem, cs>>>(a);
+      jk_kernel_ptr<X, Y>()<<<grid, 32 * WPC, smem, cs>>>(a);
     }
   }
   cudaError_t e = cudaGetLastError();
@@ -374,14 +390,15 @@ mako_status launch_batch_xy(const BatchArgs& a, void* stream) {
   using C = ClsXY<X, Y>;
   constexpr size_t smem = cta_smem_bytes<C>();
   if (a.nq <= 0) return MAKO_OK;
-  int grid = (a.nq + CTA_WARPS - 1) / CTA_WARPS;
+  int grid = (a.nq + jk_warps<C>() - 1) / jk_warps<C>();
   if (grid > 148 * 64) grid = 148 * 64;
   if constexpr (has_lowp<X, Y>()) {
     if (a.lowp && !a.diag) {
       constexpr size_t sq = cta_smem_bytes_q<C>();
       mako_status st = set_smem_attr<X, Y>((const void*)batch_kernel_q<X, Y>, sq);
       if (st) return st;
-      batch_kernel_q<X, Y><<<grid, CTA_THREADS, sq, (cudaStream_t)stream>>>(a);
+      batch_kernel_q<X, Y><<<(a.nq + q_warps<C>() - 1) / q_warps<C>() < grid ? (a.nq + q_warps<C>() - 1) / q_warps<C>() : grid,
+                             32 * q_warps<C>(), sq, (cudaStream_t)stream>>>(a);
       cudaError_t e = cudaGetLastError();
       if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("batch_kernel_q launch: ") + cudaGetErrorString(e));
       return MAKO_OK;
@@ -389,7 +406,7 @@ mako_status launch_batch_xy(const BatchArgs& a, void* stream) {
   }
   mako_status st = set_smem_attr<X, Y>((const void*)batch_kernel<X, Y>, smem);
   if (st) return st;
-  batch_kernel<X, Y><<<grid, CTA_THREADS, smem, (cudaStream_t)stream>>>(a);
+  batch_kernel<X, Y><<<grid, 32 * jk_warps<C>(), smem, (cudaStream_t)stream>>>(a);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("batch_kernel launch: ") + cudaGetErrorString(e));
   return MAKO_OK;

@@ -1,6 +1,6 @@
 // jk.cu -- mako_build_jk (the hot path), per-threshold quartet plans, sharding, eri_batch, boys.
 //
-// Plan: classes (X|Y) over pair buckets X >= Y (55 for l <= 3).  Within a
+// Plan: classes (X|Y) over pair buckets X >= Y (55 for l <= 3, 120 for l <= 4).  Within a
 // bucket pairs are sorted by Q descending, so for bra P the kets with Q_P Q_R >= thresh are a
 // PREFIX of bucket Y (clipped to R <= P when X == Y: canonical ab >= cd).  A task is (P, <= KT
 // consecutive kets of that prefix); tasks of a class are numbered by a prefix sum over P.
@@ -15,12 +15,17 @@
 namespace mako {
 
 // ----- dispatch over the 55 classes ----------------------------------------
-#define MAKO_CLASS_LIST(F)                                                                                      \
-  F(0, 0) F(1, 0) F(1, 1) F(2, 0) F(2, 1) F(2, 2) F(3, 0) F(3, 1) F(3, 2) F(3, 3) F(4, 0) F(4, 1) F(4, 2)      \
-  F(4, 3) F(4, 4) F(5, 0) F(5, 1) F(5, 2) F(5, 3) F(5, 4) F(5, 5) F(6, 0) F(6, 1) F(6, 2) F(6, 3) F(6, 4)       \
-  F(6, 5) F(6, 6) F(7, 0) F(7, 1) F(7, 2) F(7, 3) F(7, 4) F(7, 5) F(7, 6) F(7, 7) F(8, 0) F(8, 1) F(8, 2)       \
-  F(8, 3) F(8, 4) F(8, 5) F(8, 6) F(8, 7) F(8, 8) F(9, 0) F(9, 1) F(9, 2) F(9, 3) F(9, 4) F(9, 5) F(9, 6)       \
-  F(9, 7) F(9, 8) F(9, 9)
+#define MAKO_CLASS_LIST(F)                                                                                        \
+  F(0, 0) F(1, 0) F(1, 1) F(2, 0) F(2, 1) F(2, 2) F(3, 0) F(3, 1) F(3, 2) F(3, 3) F(4, 0) F(4, 1) F(4, 2)          \
+  F(4, 3) F(4, 4) F(5, 0) F(5, 1) F(5, 2) F(5, 3) F(5, 4) F(5, 5) F(6, 0) F(6, 1) F(6, 2) F(6, 3) F(6, 4)          \
+  F(6, 5) F(6, 6) F(7, 0) F(7, 1) F(7, 2) F(7, 3) F(7, 4) F(7, 5) F(7, 6) F(7, 7) F(8, 0) F(8, 1) F(8, 2)          \
+  F(8, 3) F(8, 4) F(8, 5) F(8, 6) F(8, 7) F(8, 8) F(9, 0) F(9, 1) F(9, 2) F(9, 3) F(9, 4) F(9, 5) F(9, 6)          \
+  F(9, 7) F(9, 8) F(9, 9) F(10, 0) F(10, 1) F(10, 2) F(10, 3) F(10, 4) F(10, 5) F(10, 6) F(10, 7) F(10, 8)         \
+  F(10, 9) F(10, 10) F(11, 0) F(11, 1) F(11, 2) F(11, 3) F(11, 4) F(11, 5) F(11, 6) F(11, 7) F(11, 8) F(11, 9)     \
+  F(11, 10) F(11, 11) F(12, 0) F(12, 1) F(12, 2) F(12, 3) F(12, 4) F(12, 5) F(12, 6) F(12, 7) F(12, 8) F(12, 9)    \
+  F(12, 10) F(12, 11) F(12, 12) F(13, 0) F(13, 1) F(13, 2) F(13, 3) F(13, 4) F(13, 5) F(13, 6) F(13, 7) F(13, 8)   \
+  F(13, 9) F(13, 10) F(13, 11) F(13, 12) F(13, 13) F(14, 0) F(14, 1) F(14, 2) F(14, 3) F(14, 4) F(14, 5)           \
+  F(14, 6) F(14, 7) F(14, 8) F(14, 9) F(14, 10) F(14, 11) F(14, 12) F(14, 13) F(14, 14)
 
 mako_status launch_jk_class(int X, int Y, const JKArgs& a, void* stream, int* nl) {
 #define MAKO_JK_CASE(x, y) \
@@ -217,7 +222,7 @@ __global__ void boys_kernel(int n, const double* __restrict__ T, double* __restr
     break;                                                                         \
   }
     BCASE(0) BCASE(1) BCASE(2) BCASE(3) BCASE(4) BCASE(5) BCASE(6) BCASE(7) BCASE(8) BCASE(9) BCASE(10) BCASE(11)
-    BCASE(12)
+    BCASE(12) BCASE(13) BCASE(14) BCASE(15) BCASE(16)
 #undef BCASE
   }
   for (int k = 0; k <= mmax; ++k) out[(size_t)i * (mmax + 1) + k] = F[k];
@@ -461,7 +466,7 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
     if (mixed && (st = ensure_lowp(p->set, cuda_stream))) return st;
     if ((st = cuda_check(cudaMemsetAsync(J, 0, sizeof(double) * n * n, s), "memset J")) ||
         (st = cuda_check(cudaMemsetAsync(K, 0, sizeof(double) * n * n, s), "memset K")) ||
-        (st = cuda_check(cudaMemsetAsync(p->d_counters.p, 0, sizeof(unsigned long long) * 128, s), "memset ctr")))
+        (st = cuda_check(cudaMemsetAsync(p->d_counters.p, 0, sizeof(unsigned long long) * 2 * NCLASS, s), "memset ctr")))
       return st;
     int nl = 0;
     if ((st = ensure_streams(p))) return st;
@@ -470,7 +475,7 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
     for (void* is : p->streams) cudaStreamWaitEvent((cudaStream_t)is, (cudaEvent_t)p->ev_fork, 0);
     // classes in descending estimated cost, greedily balanced over the internal streams; each kernel
     // gets half of the resident capacity so two classes (often a DFMA- and a DMMA-bound one) co-reside
-    // (index >= 55: the class's TF32-tier plan)
+    // (index >= NCLASS: the class's TF32-tier plan)
     const int NCL = (int)p->plan.cls.size();
     std::vector<std::pair<double, int>> order;
     for (int i = 0; i < (mixed ? 2 * NCL : NCL); ++i) {

@@ -20,7 +20,8 @@
 namespace mako {
 
 constexpr int LMAX = MAKO_LMAX;
-constexpr int NBUCKET = (LMAX + 1) * (LMAX + 2) / 2;  // (la >= lb) pair classes: ss ps pp ds dp dd fs fp fd ff
+constexpr int NBUCKET = (LMAX + 1) * (LMAX + 2) / 2;  // (la >= lb) pair buckets: ss ps pp ds dp dd fs fp fd ff gs gp gd gf gg
+constexpr int NCLASS = NBUCKET * (NBUCKET + 1) / 2;
 
 // number of Hermite (or Cartesian) tuples (t,u,v) with t+u+v <= L
 MK_HD constexpr int nH(int L) { return L < 0 ? 0 : (L + 1) * (L + 2) * (L + 3) / 6; }
@@ -55,14 +56,18 @@ constexpr size_t BOYS_TABLE_DOUBLES = BOYS_EXP_OFF + BOYS_NEXP;
 // Kernel family per class (X >= Y buckets).  Low-l classes use the lane-per-ket register kernel
 // ("TPQ": Boys, R, contraction and digestion in registers of one lane), the rest the warp-per-quartet
 // DMMA kernel.  Register estimate (doubles): R + V + W + cached ket E~ + cached bra E~.
-MK_HD constexpr int b_la(int b) { return b >= 6 ? 3 : (b >= 3 ? 2 : (b >= 1 ? 1 : 0)); }
+MK_HD constexpr int b_la(int b) {  // bucket b = la (la + 1) / 2 + lb
+  int la = 0;
+  while ((la + 1) * (la + 2) / 2 <= b) ++la;
+  return la;
+}
 MK_HD constexpr int b_lb(int b) { return b - b_la(b) * (b_la(b) + 1) / 2; }
 MK_HD constexpr int tpq_regs(int X, int Y) {
   return nH(b_la(X) + b_lb(X) + b_la(Y) + b_lb(Y)) + nsph(b_la(X)) * nsph(b_lb(X)) * nsph(b_la(Y)) * nsph(b_lb(Y)) +
          nsph(b_la(Y)) * nsph(b_lb(Y)) * (1 + nH(b_la(Y) + b_lb(Y))) +
          (nsph(b_la(X)) * nsph(b_lb(X)) * nH(b_la(X) + b_lb(X)) <= 40 ? nsph(b_la(X)) * nsph(b_lb(X)) * nH(b_la(X) + b_lb(X)) : 0);
 }
-MK_HD constexpr bool use_tpq(int X, int Y) { return Y <= 1 && tpq_regs(X, Y) <= 100; }
+MK_HD constexpr bool use_tpq(int X, int Y) { return Y <= 1 && b_la(X) <= 3 && tpq_regs(X, Y) <= 100; }
 MK_HD constexpr int class_kt(int X, int Y) { return use_tpq(X, Y) ? 32 : 16; }
 
 // reduced-precision tier: floats per primitive pair of the TF32 fragment-order copies of E~ (pairs.cu

@@ -98,7 +98,7 @@ struct mako_pairs_s {
   mako::PairSet set;
   mako::Plan plan;                       // current plan
   std::vector<mako::Plan> plan_cache;    // recently used plans of other thresholds (density screening)
-  mako::DevBuf d_counters;      // [55] task counters
+  mako::DevBuf d_counters;      // [2 * NCLASS] task counters (FP64 tier, TF32 tier)
   mako::DevBuf d_dsh;           // [nshell * nshell] float: max |D| per shell block (density screening)
   mako::DevBuf d_dmax;          // [1] double: max |D| (density screening)
   // profiling (mako_profile_enable / read)

@@ -342,7 +342,7 @@ extern "C" mako_status mako_shellpairs_screen(mako_basis basis, double thresh, v
       P->set.b[b].seg = seg[b];
       if ((st = upload_async(P->set.b[b].d_Q, Q2[b], s))) return st;
     }
-    if ((st = P->d_counters.alloc(sizeof(unsigned long long) * 128))) return st;
+    if ((st = P->d_counters.alloc(sizeof(unsigned long long) * 2 * NCLASS))) return st;
     if ((st = cuda_check(cudaStreamSynchronize(s), "screen sync"))) return st;
     *out = P.release();
     return MAKO_OK;

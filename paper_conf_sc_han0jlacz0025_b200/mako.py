@@ -162,7 +162,7 @@ def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=N
 
 
 def class_reduced():
-    """[55] bool: classes with a reduced-precision (TF32) kernel (mako_class_reduced)."""
+    """[MAKO_NCLASS] bool: classes with a reduced-precision (TF32) kernel (mako_class_reduced)."""
     m = np.zeros(_lib.NCLASS, np.int32)
     check(_lib.load().mako_class_reduced(m.ctypes.data_as(ctypes.POINTER(ctypes.c_int))))
     return m.astype(bool)

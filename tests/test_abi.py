@@ -31,13 +31,21 @@ def test_library_exports_every_header_symbol():
     assert b"sm_100a" in lib.mako_version()
 
 
+def _sass(function):
+    """SASS of one kernel of the library (cuobjdump -fun; the whole 60+ MB dump takes a minute)."""
+    import subprocess
+    from paper_conf_sc_han0jlacz0025_b200 import _lib
+    return subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", "-fun", function, _lib.LIB_PATH],
+                          capture_output=True, text=True).stdout
+
+
 def test_library_is_sm100a_cubin():
     import subprocess
     from paper_conf_sc_han0jlacz0025_b200 import _lib
     out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", _lib.LIB_PATH], capture_output=True, text=True)
     assert "sm_100a" in out.stdout
-    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", _lib.LIB_PATH], capture_output=True, text=True).stdout
-    assert "DMMA" in sass  # FP64 tensor-core MMA (mma.sync .f64) in the class kernels
+    # FP64 tensor-core MMA (mma.sync .f64) in the (ff|ff) class kernel
+    assert "DMMA" in _sass("_ZN4mako14jk_kernel_freeILi9ELi9ELb0EEEvNS_6JKArgsE")
 
 
 def test_errors_without_gpu():
@@ -68,13 +76,12 @@ def test_reduced_precision_tier_boundary():
     """the TF32 tier exists in the library (SASS HMMA.1688.F32.TF32 next to DMMA), covers
     every high-l class (L >= 8, where the basis transformation dominates), and the mixed build
     validates its arguments before touching the device."""
-    import subprocess
     from paper_conf_sc_han0jlacz0025_b200 import _lib, class_reduced
-    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", _lib.LIB_PATH], capture_output=True, text=True).stdout
-    assert "HMMA.1688.F32.TF32" in sass
+    assert "HMMA.1688.F32.TF32" in _sass("_ZN4mako11jk_kernel_qILi9ELi9ELb0EEEvNS_6JKArgsE")
+    assert "HMMA.1688.F32.TF32" in _sass("_ZN4mako11jk_kernel_qILi14ELi14ELb0EEEvNS_6JKArgsE")  # (gg|gg)
     m = class_reduced()
-    bl = [(0, 0), (1, 0), (1, 1), (2, 0), (2, 1), (2, 2), (3, 0), (3, 1), (3, 2), (3, 3)]
-    for X in range(10):
+    bl = [(la, lb) for la in range(5) for lb in range(la + 1)]
+    for X in range(15):
         for Y in range(X + 1):
             if sum(bl[X]) + sum(bl[Y]) >= 8:
                 assert m[X * (X + 1) // 2 + Y], (bl[X], bl[Y])

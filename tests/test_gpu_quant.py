@@ -21,7 +21,7 @@ import mako_inputs as mi
 
 pytestmark = pytest.mark.gpu
 
-NAMES = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff"]
+NAMES = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff", "gs", "gp", "gd", "gf", "gg"]
 
 
 def _bucket(la, lb):
