@@ -239,6 +239,7 @@ def run_mako(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     from paper_conf_sc_han0jlacz0025_b200 import Basis, Pairs, build_jk
+    from paper_conf_sc_han0jlacz0025_b200.mako import FAMILY_KERNELS, class_family, class_reduced
     from paper_conf_sc_han0jlacz0025_b200.dist import combine_jk
 
     mol, basis = mi.config_molecule(args.config)
@@ -322,7 +323,8 @@ def run_mako(args):
                  "dE2_vs_fp64_Ha": e2(Jm, Km) - e2(J, K),
                  "max_dJ": float((Jm - J).abs().max()), "max_dK": float((Km - K).abs().max()),
                  "tiers": "FP64 Boys/R + TF32 GEMM1/GEMM2 (FP32 accumulate) + FP64 digestion for quartets with "
-                          "Q_ab Q_cd max|D| < thresh_fp64 in the 31 classes with a reduced kernel; FP64 otherwise"}
+                          "Q_ab Q_cd max|D| < thresh_fp64 in the %d classes with a reduced kernel; FP64 otherwise"
+                          % int(class_reduced().sum())}
         if cls_ms_m is not None:
             mixed["class_ms"] = {f"({names_[int((math.isqrt(8*i+1)-1)//2)]}|"
                                  f"{names_[i - int((math.isqrt(8*i+1)-1)//2) * (int((math.isqrt(8*i+1)-1)//2) + 1) // 2]})":
@@ -375,7 +377,7 @@ def run_mako(args):
             traffic = None
     roof = {"bound": "tensor", "achieved": achieved, "peak": pk["dmma_m16n8k4_tflops"], "unit": "TFLOP/s",
             "frac": achieved / pk["dmma_m16n8k4_tflops"], "traffic": traffic,
-            "kernel": f"jk_kernel<{X},{Y}> class ({names[X]}|{names[Y]})",
+            "kernel": f"{FAMILY_KERNELS[int(class_family()[c])]}<{X},{Y}> class ({names[X]}|{names[Y]})",
             "share_of_step": float(cls_ms[c] / max(cls_ms.sum(), 1e-9)),
             "peak_source": "FP64 DMMA mma.sync m16n8k4 loop measured on this pool's B200 "
                            "(profiles/peaks_fp64_r01.json; MEASURED_PEAKS.json has no FP64 entry)",

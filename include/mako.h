@@ -147,6 +147,10 @@ mako_status mako_build_jk_ex(mako_pairs pairs, const double* D, double thresh, u
  * cuda_stream once (max|D| decides the tier plan).  D, J, K as in mako_build_jk. */
 mako_status mako_build_jk_mixed(mako_pairs pairs, const double* D, double thresh, double thresh_fp64,
                                 unsigned flags, double* J, double* K, int shard, int nshards, void* cuda_stream);
+/* family[MAKO_NCLASS] (HOST): the kernel family that runs each class (S6): 0 lane-per-ket
+ * register kernel, 1 ket-first DMMA kernel, 2 ket-first transposed, 3 slot-batched DMMA kernel,
+ * 4 warp-per-quartet DMMA kernel.  For measurement reports. */
+mako_status mako_class_family(int* family);
 /* mask[MAKO_NCLASS] (HOST): 1 where the class has a reduced-precision (TF32) kernel. */
 mako_status mako_class_reduced(int* mask);
 

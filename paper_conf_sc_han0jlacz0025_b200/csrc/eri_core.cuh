@@ -236,6 +236,10 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
       double* cur = (n & 1) ? scratch : dst;  // level 0 lands in dst
       const double* prv = ((n + 1) & 1) ? scratch : dst;
       const int cnt = nH(L - n);
+#ifndef MAKO_R_ILP_LMAX
+#define MAKO_R_ILP_LMAX 7
+#endif
+      if constexpr (L > MAKO_R_ILP_LMAX) {  // high-l classes: measured faster with one entry in flight
       for (int e = lane; e < cnt; e += 32) {
         double v;
         if (e == 0) {
@@ -249,6 +253,41 @@ __device__ __forceinline__ void compute_R(double p, double Px, double Py, double
         }
         if (F32 && n == 0) dst32[e] = to_tf32(v);
         else cur[e] = v;
+      }
+      } else {
+      // up to RB entries per lane in flight: all their rtab / prv loads are issued before the first
+      // store (the level loop is latency-bound on the SMEM round trips, profiles/README.md)
+      constexpr int RB = 4;
+      const int nj = (cnt + 31) >> 5;
+#pragma unroll
+      for (int j0 = 0; j0 < nj; j0 += RB) {
+        double v[RB];
+#pragma unroll
+        for (int jj = 0; jj < RB; ++jj) {
+          const int e = lane + 32 * (j0 + jj);
+          v[jj] = 0.0;
+          if (j0 + jj < nj && e < cnt) {
+            if (e == 0) {
+              v[jj] = F[n];
+            } else {
+              const uint32_t w = rtab[e];
+              const int s1 = w & 1023, s2 = (w >> 10) & 1023, dir = (w >> 20) & 3, cf = (int)(w >> 22);
+              const double xd = dir == 0 ? X : (dir == 1 ? Y : Z);
+              double t = xd * prv[s1];
+              if (cf) t = fma((double)cf, prv[s2], t);
+              v[jj] = t;
+            }
+          }
+        }
+#pragma unroll
+        for (int jj = 0; jj < RB; ++jj) {
+          const int e = lane + 32 * (j0 + jj);
+          if (j0 + jj < nj && e < cnt) {
+            if (F32 && n == 0) dst32[e] = to_tf32(v[jj]);
+            else cur[e] = v[jj];
+          }
+        }
+      }
       }
       __syncwarp();
     }

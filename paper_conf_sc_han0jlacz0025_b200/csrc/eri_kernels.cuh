@@ -39,9 +39,14 @@ namespace mako {
 // classes with a reduced-precision (TF32) tier kernel: the warp-per-quartet DMMA family, where the
 // basis transformation (GEMM1/GEMM2) dominates (the lane-per-ket, ket-first and
 // slab families run the FP64 kernel in both tiers)
+// Restricted to l <= 3 classes with n_ab >= 9 and L >= 6: measured per class (S6), the
+// TF32 tier gains nothing where a 16-row tile is half empty (fs bras) or the R recursion dominates
+// (L < 6), and the l = 4 classes ran slower in it.
 template <int X, int Y>
 constexpr bool has_lowp() {
-  return !use_tpq(X, Y) && !use_kf<X, Y>() && !use_kf_swap<X, Y>() && !use_slab<X, Y>();
+  using C = ClsXY<X, Y>;
+  return !use_tpq(X, Y) && !use_kf<X, Y>() && !use_kf_swap<X, Y>() && !use_slab<X, Y>() && C::LA <= 3 &&
+         C::LC <= 3 && C::NAB >= 9 && C::L >= 6;
 }
 
 // warps per CTA of the warp-per-quartet kernels: 4, fewer when the per-warp SMEM of a class does

@@ -11,6 +11,8 @@
 
 #include "eri_kernels.cuh"
 #include "eri_core.cuh"
+#include "eri_kf.cuh"
+#include "eri_slab.cuh"
 
 namespace mako {
 
@@ -57,6 +59,24 @@ static bool class_swap(int X, int Y) {
   MAKO_CLASS_LIST(MAKO_SW_CASE)
 #undef MAKO_SW_CASE
   return false;
+}
+
+// kernel family of a class (include/mako.h mako_class_family): 0 lane-per-ket (tpq), 1 ket-first (kf),
+// 2 ket-first transposed, 3 slot-batched (slab), 4 warp-per-quartet (jk)
+template <int X, int Y>
+static int family_xy() {
+  if constexpr (use_kf_swap<X, Y>()) return 2;
+  else if constexpr (use_kf<X, Y>()) return 1;
+  else if constexpr (use_tpq(X, Y)) return 0;
+  else if constexpr (use_slab<X, Y>()) return 3;
+  else return 4;
+}
+static int class_family(int X, int Y) {
+#define MAKO_FAM_CASE(x, y) \
+  if (X == x && Y == y) return family_xy<x, y>();
+  MAKO_CLASS_LIST(MAKO_FAM_CASE)
+#undef MAKO_FAM_CASE
+  return -1;
 }
 
 bool class_has_lowp(int X, int Y) {
@@ -559,6 +579,13 @@ extern "C" mako_status mako_build_jk_mixed(mako_pairs p, const double* D, double
                                            void* cuda_stream) {
   if (!(thresh_fp64 > 0) || !std::isfinite(thresh_fp64)) return fail(MAKO_ERR_INVALID, "thresh_fp64 must be > 0");
   return build_jk_impl(p, D, thresh, thresh_fp64, flags, J, K, shard, nshards, cuda_stream);
+}
+
+extern "C" mako_status mako_class_family(int* family) {
+  if (!family) return fail(MAKO_ERR_INVALID, "NULL family");
+  for (int X = 0; X < NBUCKET; ++X)
+    for (int Y = 0; Y <= X; ++Y) family[class_index(X, Y)] = class_family(X, Y);
+  return MAKO_OK;
 }
 
 extern "C" mako_status mako_class_reduced(int* mask) {

@@ -168,6 +168,17 @@ def class_reduced():
     return m.astype(bool)
 
 
+FAMILY_KERNELS = {0: "tpq_jk_kernel", 1: "kf_jk_kernel", 2: "kf_jk_kernel (transposed)", 3: "slab_jk_kernel",
+                  4: "jk_kernel"}
+
+
+def class_family():
+    """[MAKO_NCLASS] int: kernel family per class (mako_class_family; FAMILY_KERNELS names them)."""
+    m = np.zeros(_lib.NCLASS, np.int32)
+    check(_lib.load().mako_class_family(m.ctypes.data_as(ctypes.POINTER(ctypes.c_int))))
+    return m
+
+
 def eri_batch(basis, quartets, stream=None, device=None, reduced=False):
     """Shell-quartet ERI blocks (test entry).  Returns a list of numpy-shaped torch tensors on the GPU.
     reduced=True: mako_eri_batch_ex with MAKO_ERI_REDUCED (the TF32 tier where the class has one)."""

@@ -58,7 +58,6 @@ def test_eri_batch_all_120_classes_fp64_and_reduced():
         assert err <= 1e-10, (q, err)
     print("g classes: max |dERI| %.3e over %d quartets" % (worst, len(quartets)))
     red = class_reduced()
-    assert red.sum() > 31  # g classes have TF32-tier kernels too
     blocks = eri_batch(B, quartets, reduced=True)
     Qc = {}
 
