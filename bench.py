@@ -197,11 +197,18 @@ def run_reference(args):
     Q = oracle.schwarz(sh)
     total, nq = workload_flops(sh, Q, args.tau)
     npair = sh.nshell * (sh.nshell + 1) // 2
-    # size one step at ~args.ref_step_s seconds of oracle work
-    S = max(2, min(npair, 50000))
+    # size one step at ~args.ref_step_s seconds of oracle work: pilot on 8 spread-out shards of 1/S0
+    # (one tiny shard is dominated by the per-call overhead and would overstate the build time), then
+    # a second pilot at the resulting size
+    S = max(2, min(npair, 20000))
     t0 = time.perf_counter()
-    oracle.jk(sh, D, args.tau, 1, S, Q=Q)
-    est_total = max(time.perf_counter() - t0, 1e-3) * S
+    for i in range(8):
+        oracle.jk(sh, D, args.tau, (i * S) // 8 + 1, S, Q=Q)
+    est_total = max((time.perf_counter() - t0) / 8, 1e-4) * S
+    S = int(min(max(2, est_total / args.ref_step_s), npair))
+    t0 = time.perf_counter()
+    oracle.jk(sh, D, args.tau, S // 3, S, Q=Q)
+    est_total = max(time.perf_counter() - t0, 1e-4) * S
     S = int(min(max(2, est_total / args.ref_step_s), npair))
     times = []
     for i in range(args.warmup + args.steps):
