@@ -119,6 +119,7 @@ static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const Pa
   c.kbeg.clear();
   c.kend.clear();
   c.task_off.assign(1, 0);
+  c.cost_cum.assign(1, 0.0);
   c.nquartet = 0;
   for (int p = 0; p < nbra; ++p)
     for (int g = 0; g < G; ++g) {
@@ -136,6 +137,8 @@ static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const Pa
       c.kend.push_back(s0 + nk);
       c.nquartet += nk - nh;
       c.task_off.push_back(c.task_off.back() + (nk - nh + c.KT - 1) / c.KT);
+      c.cost_cum.push_back(c.cost_cum.back() + (double)(bx.poff[p + 1] - bx.poff[p]) *
+                                                   (double)(by.poff[s0 + nk] - by.poff[s0 + nh]));
     }
   c.ntask = c.task_off.back();
   c.usamp.assign((size_t)(c.ntask >> TASK_SAMPLE_SHIFT) + 1, 0);
@@ -150,6 +153,24 @@ static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const Pa
                       (st = upload(c.d_usamp, c.usamp))))
     return st;
   return MAKO_OK;
+}
+
+// Task index of the cut between shard s-1 and shard s of n (s = 0..n) in class plan c:
+// contiguous ranges of EQUAL COST, cost = primitive quartets (K_task-pair x sum K of its kets), cut
+// inside an entry in proportion to its tasks.  A pure function of the plan, monotone in s.
+static long long shard_cut(const ClassPlan& c, int s, int n) {
+  if (s <= 0 || c.ntask == 0) return 0;
+  if (s >= n) return c.ntask;
+  const double total = c.cost_cum.back();
+  if (!(total > 0)) return c.ntask * s / n;
+  const double target = total * s / n;
+  size_t u = std::upper_bound(c.cost_cum.begin(), c.cost_cum.end(), target) - c.cost_cum.begin();
+  u = u == 0 ? 0 : u - 1;
+  if (u + 1 >= c.cost_cum.size()) return c.ntask;
+  const double w = c.cost_cum[u + 1] - c.cost_cum[u];
+  const long long nt = c.task_off[u + 1] - c.task_off[u];
+  const long long k = w > 0 ? std::llround((target - c.cost_cum[u]) / w * (double)nt) : 0;
+  return c.task_off[u] + std::min(std::max(k, 0LL), nt);
 }
 
 // Plan for Schwarz threshold `thresh`; with tier > thresh (reduced-precision build)
@@ -304,7 +325,7 @@ static mako_status class_flops(mako_pairs p, double thresh, int shard, int nshar
     const int la = bucket_la(c.X), lb = bucket_lb(c.X), lc = bucket_la(c.Y), ld = bucket_lb(c.Y);
     const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
     const double hab = nH(la + lb), hcd = nH(lc + ld);
-    const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
+    const long long t0 = shard_cut(c, shard, nshards), t1 = shard_cut(c, shard + 1, nshards);
     // surviving kets of each (bra, K-group) entry restricted to this shard's tasks
     for (size_t u = 0; u < c.kbeg.size(); ++u) {
       const long long a0 = c.task_off[u], a1 = c.task_off[u + 1];
@@ -434,7 +455,7 @@ extern "C" mako_status mako_build_jk_launches(mako_pairs p, double thresh, int s
   if ((st = ensure_plan(p, thresh))) return st;
   int cnt = 1;  // symmetrize
   for (auto& c : p->plan.cls) {
-    const long long t0 = c.ntask * shard / nshards, t1 = c.ntask * (shard + 1) / nshards;
+    const long long t0 = shard_cut(c, shard, nshards), t1 = shard_cut(c, shard + 1, nshards);
     if (t1 > t0) ++cnt;
   }
   *n = cnt;
@@ -511,8 +532,8 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
       const bool lo = oc.second >= NCL;
       ClassPlan& c = lo ? p->plan.cls_lo[oc.second - NCL] : p->plan.cls[oc.second];
       JKArgs a{};
-      a.task_begin = c.ntask * shard / nshards;
-      a.task_end = c.ntask * (shard + 1) / nshards;
+      a.task_begin = shard_cut(c, shard, nshards);
+      a.task_end = shard_cut(c, shard + 1, nshards);
       if (a.task_end <= a.task_begin) continue;
       const size_t si = std::min_element(load.begin(), load.end()) - load.begin();
       load[si] += -oc.first;
