@@ -108,8 +108,9 @@ void mako_pairs_destroy(mako_pairs pairs);
  *         this shard that survive Q_ab Q_cd >= thresh.  Both come out exactly symmetric.
  *   thresh >= the pairs' screening threshold (smaller values are treated as equal to it).
  *   shard, nshards: 0 <= shard < nshards.  The canonical quartet tasks of every angular-momentum
- *         class are split into nshards contiguous ranges of equal cost (primitive quartets; SURVEY
- *         S8.e); shard `shard` takes its range.
+ *         class are split into nshards contiguous ranges of equal modelled cost (primitive quartets,
+ *         ket primitive pairs and quartets, weighted by the class's work per unit);
+ *         shard `shard` takes its range.
  *         A pure function of (pairs, thresh, shard, nshards): summing J/K over all shards gives the
  *         nshards = 1 result up to FP64 summation order.
  *   cuda_stream: all work is enqueued on it (async).  J, K, D must not alias. */

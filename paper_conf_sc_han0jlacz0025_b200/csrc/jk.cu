@@ -115,6 +115,15 @@ static int prefix_count(const std::vector<double>& QY, int lo0, int hi0, double 
 static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const PairBucket& by, bool same, double lo,
                                     double hi) {
   const int nbra = bx.n(), G = NKGROUP;
+  // shard-balance cost model of one quartet of this class (FLOP-like units): per primitive
+  // quartet the Boys seed + R recursion + GEMM1 row, per ket primitive pair GEMM2, per quartet the
+  // digestion and task overhead.  Measured: primitive quartets alone left shard 0 (many K = 1 bras)
+  // 25 % above the mean on the valinomycin build.
+  const int la = bx.la, lb = bx.lb, lc = by.la, ld = by.lb, L = la + lb + lc + ld;
+  const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
+  const double cA = 2.0 * nab * nH(la + lb) * nH(lc + ld) + 4.0 * nH(L) * (L + 1) + 60.0;
+  const double cB = 2.0 * nab * nH(lc + ld) * ncd;
+  const double cC = 12.0 * nab * ncd + 200.0;
   c.ent_P.clear();
   c.kbeg.clear();
   c.kend.clear();
@@ -137,8 +146,8 @@ static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const Pa
       c.kend.push_back(s0 + nk);
       c.nquartet += nk - nh;
       c.task_off.push_back(c.task_off.back() + (nk - nh + c.KT - 1) / c.KT);
-      c.cost_cum.push_back(c.cost_cum.back() + (double)(bx.poff[p + 1] - bx.poff[p]) *
-                                                   (double)(by.poff[s0 + nk] - by.poff[s0 + nh]));
+      const double kab = bx.poff[p + 1] - bx.poff[p], skcd = by.poff[s0 + nk] - by.poff[s0 + nh];
+      c.cost_cum.push_back(c.cost_cum.back() + kab * skcd * cA + skcd * cB + (nk - nh) * cC);
     }
   c.ntask = c.task_off.back();
   c.usamp.assign((size_t)(c.ntask >> TASK_SAMPLE_SHIFT) + 1, 0);
@@ -156,8 +165,8 @@ static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const Pa
 }
 
 // Task index of the cut between shard s-1 and shard s of n (s = 0..n) in class plan c:
-// contiguous ranges of EQUAL COST, cost = primitive quartets (K_task-pair x sum K of its kets), cut
-// inside an entry in proportion to its tasks.  A pure function of the plan, monotone in s.
+// contiguous ranges of EQUAL COST (the cost model of build_class_plan), cut inside an entry in
+// proportion to its tasks.  A pure function of the plan, monotone in s.
 static long long shard_cut(const ClassPlan& c, int s, int n) {
   if (s <= 0 || c.ntask == 0) return 0;
   if (s >= n) return c.ntask;

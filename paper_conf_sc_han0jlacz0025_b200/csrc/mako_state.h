@@ -66,7 +66,7 @@ struct ClassPlan {
   std::vector<int> ent_P, kbeg, kend;  // [nent] bra pair, first / one-past-last surviving ket
   std::vector<long long> task_off;     // [nent + 1] task prefix
   std::vector<int> usamp;              // [ntask / TASK_SAMPLE + 1] entry holding task k * TASK_SAMPLE
-  std::vector<double> cost_cum;        // [nent + 1] prefix of primitive quartets per entry (shard balance)
+  std::vector<double> cost_cum;        // [nent + 1] prefix of the modelled cost per entry (shard balance)
   DevBuf d_ent_P, d_kbeg, d_kend, d_task_off, d_usamp;
 };
 
