@@ -151,3 +151,32 @@ def test_flop_accounting_library_equals_reference_arm():
     py_flops, py_q = bench.workload_flops(sh, oracle.schwarz(sh), 1e-12)
     assert py_q == lib["quartets"]
     assert abs(py_flops - lib["gemm_flops"]) <= 1e-9 * lib["gemm_flops"]
+
+
+def _contracted_basis(centers, k, seed):
+    """Random centres with one s, p, d and f shell each, k primitives on every shell (the paper's E1
+    setting): the d/f x d/f bras are contracted, so the chunk-outer kernels
+    (jk_kernel_cb, quartet_block_cbra) run."""
+    rng = np.random.default_rng(seed)
+    xyz = rng.uniform(-1.5, 1.5, size=(centers, 3))
+    at, ls, nps, ex, cf = [], [], [], [], []
+    for a in range(centers):
+        for l in range(4):
+            at.append(a); ls.append(l); nps.append(k)
+            ex += list(np.sort(np.exp(rng.uniform(np.log(0.2), np.log(5.0), k)))[::-1])
+            cf += list(rng.uniform(0.2, 1.0, k))
+    sh = mi.Shells(np.array(at, np.int32), np.array(ls, np.int32), np.array(nps, np.int32), xyz[np.array(at)],
+                   np.array(ex), np.array(cf))
+    return sh, np.ones(centers, np.int32), xyz
+
+
+def test_contracted_df_bras_vs_oracle():
+    from paper_conf_sc_han0jlacz0025_b200 import Basis, Pairs
+    sh, Z, xyz = _contracted_basis(3, 3, seed=11)
+    P = Pairs(Basis(Z, xyz, sh), 0.0)
+    D = mi.synthetic_density(sh.nbf(), 6, seed=3)
+    J0, K0 = oracle.jk(sh, D, 0.0)
+    J, K = _gpu_jk(P, D)
+    dj, dk = np.abs(J - J0).max(), np.abs(K - K0).max()
+    print("contracted d/f max|dJ|", dj, "max|dK|", dk, "|J|", np.abs(J0).max())
+    assert dj <= 1e-8 and dk <= 1e-8
