@@ -219,11 +219,13 @@ static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0) {
         const double lo = part ? thresh : (split ? tier : thresh), hi = part ? tier : inf;
         mako_status st = build_class_plan(c, P->set.b[c.TB], P->set.b[c.LB], X == Y, lo, hi);
         if (st) return st;
-        // warp-per-quartet classes with few quartets (contracted or small high-l workloads, e.g. the
-        // paper's E1 microbenchmark): shorter tasks so that the 148 SMs see at
-        // least ~32 grabs (TASK_GRAB tasks each) per SM instead of a few long-running warps
+        // warp-per-quartet and slot-batched classes (runtime KT) with few quartets (contracted or small
+        // high-l workloads, e.g. the paper's E1 microbenchmark): shorter tasks so
+        // that the 148 SMs see at least ~32 grabs (TASK_GRAB tasks each) per SM instead of a few
+        // long-running warps
         const long long want = (long long)TASK_GRAB * 148 * 32;
-        if (class_family(X, Y) == 4 && c.nquartet > 0 && c.nquartet / c.KT < want) {
+        const int fam = class_family(X, Y);
+        if ((fam == 4 || fam == 3) && c.nquartet > 0 && c.nquartet / c.KT < want) {
           c.KT = (int)std::max<long long>(1, c.nquartet / want);
           if ((st = build_class_plan(c, P->set.b[c.TB], P->set.b[c.LB], X == Y, lo, hi))) return st;
         }
