@@ -7,6 +7,7 @@
 // Sharding: shard s of n takes tasks [T s/n, T (s+1)/n) of every class.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <limits>
 
 #include "eri_kernels.cuh"
@@ -182,6 +183,8 @@ static long long shard_cut(const ClassPlan& c, int s, int n) {
   return c.task_off[u] + std::min(std::max(k, 0LL), nt);
 }
 
+constexpr int KT_JK = 4;
+
 // Plan for Schwarz threshold `thresh`; with tier > thresh (reduced-precision build)
 // the quartets of classes that have a TF32-tier kernel are split: Q_ab Q_cd >= tier into cls (FP64),
 // thresh <= Q_ab Q_cd < tier into cls_lo (TF32).  tier = 0: one FP64 tier.
@@ -213,6 +216,15 @@ static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0) {
         c.X = X;
         c.Y = Y;
         c.KT = class_task_kets(X, Y);
+        // warp-per-quartet classes: 4 kets per task (measured on the bench workload, tools/exp/kt.sh:
+        // family time 5.60 / 5.52 / 5.47 / 5.45 s at KT = 32 / 16 / 8 / 4; the slot-batched kernel
+        // batches ket primitives across the kets of a task and keeps 16)
+        if (class_family(X, Y) == 4) c.KT = KT_JK;
+        {  // experiments only (tools/exp): MAKO_KT_EXP overrides the base task length of the runtime-KT families
+          static const int kt_exp = std::getenv("MAKO_KT_EXP") ? std::atoi(std::getenv("MAKO_KT_EXP")) : 0;
+          const int f = class_family(X, Y);
+          if (kt_exp > 0 && (f == 3 || f == 4)) c.KT = kt_exp;
+        }
         c.swap = class_swap(X, Y);
         c.TB = c.swap ? Y : X;
         c.LB = c.swap ? X : Y;
