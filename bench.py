@@ -159,33 +159,67 @@ class ClockSampler:
 # ---------------------------------------------------------------------------------------------
 # CPU baseline: the oracle as it stands, on a bounded sample of the same workload
 # ---------------------------------------------------------------------------------------------
+def oracle_overhead(sh, D, tau, Q):
+    """Per-call cost of oracle.jk that does not scale with the sample (per-thread nbf^2 accumulators,
+    their reduction, the symmetrisation): one call on an empty shard (no bra pair has index % S == S-1
+    when S > npair).  A full build pays it once."""
+    import oracle
+    npair = sh.nshell * (sh.nshell + 1) // 2
+    t0 = time.perf_counter()
+    oracle.jk(sh, D, tau, npair, npair + 1, Q=Q)
+    return time.perf_counter() - t0
+
+
+def oracle_sample_seconds(sh, D, tau, Q, target_s, first_shard=0):
+    """Size a strided sample of canonical bra pairs (index % S == shard) so that its WORK (call time
+    minus the per-call overhead) is about target_s; returns (S, overhead_s).  The pilot uses 8 spread
+    shards of 1/S0 so that one atypical pair does not set the size."""
+    import oracle
+    npair = sh.nshell * (sh.nshell + 1) // 2
+    ovh = oracle_overhead(sh, D, tau, Q)
+    S0 = max(2, min(npair, 20000))
+    t0 = time.perf_counter()
+    for i in range(8):
+        oracle.jk(sh, D, tau, (first_shard + (i * S0) // 8 + 1) % S0, S0, Q=Q)
+    work = max((time.perf_counter() - t0) / 8 - ovh, 1e-4)
+    S = int(min(work * S0 / target_s, npair))  # S < 2: the full build fits the budget
+    return S, ovh
+
+
+def oracle_sampled_build(sh, D, tau, Q, S, shard, ovh):
+    """One timed oracle call on the sample shard/S; extrapolated full-build seconds
+    (work x S + the per-call overhead once)."""
+    import oracle
+    t0 = time.perf_counter()
+    oracle.jk(sh, D, tau, shard, S, Q=Q)
+    ts = time.perf_counter() - t0
+    return ts, max(ts - ovh, 0.0) * S + ovh
+
+
 def cpu_baseline(sh, D, tau, total_flops, target_s=15.0, Q=None):
     import oracle
     if Q is None:
         Q = oracle.schwarz(sh)
-    # pilot on 8 spread-out tiny shards, then size the sample to ~target_s
-    npair = sh.nshell * (sh.nshell + 1) // 2
-    S = max(2, min(npair, 20000))
-    t0 = time.perf_counter()
-    for i in range(8):
-        oracle.jk(sh, D, tau, (i * S) // 8 + 1, S, Q=Q)
-    tp = (time.perf_counter() - t0) / 8
-    est_total = max(tp, 1e-4) * S
-    S = int(min(max(2, est_total / target_s), npair))
+    S, ovh = oracle_sample_seconds(sh, D, tau, Q, target_s)
+    if S < 2:  # the whole build fits the budget: time it directly
+        t0 = time.perf_counter()
+        oracle.jk(sh, D, tau, Q=Q)
+        ts = time.perf_counter() - t0
+        return {"value": total_flops / ts / 1e12, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+                "sample": f"the full build, {ts:.1f} s", "s_per_iter": ts, "extrapolated": False}
     shard = S // 2
-    t0 = time.perf_counter()
-    oracle.jk(sh, D, tau, shard, S, Q=Q)
-    ts = time.perf_counter() - t0
-    s_per_build = ts * S
+    ts, s_per_build = oracle_sampled_build(sh, D, tau, Q, S, shard, ovh)
     return {"value": total_flops / s_per_build / 1e12, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"canonical bra pairs with pair_index % {S} == {shard} (1/{S} of the build), "
-                      f"{ts:.1f} s, extrapolated x{S}",
-            "s_per_iter_extrapolated": s_per_build}
+            "sample": f"canonical bra pairs with pair_index % {S} == {shard} (1/{S} of the build): {ts:.1f} s "
+                      f"measured, per-call overhead {ovh:.2f} s (empty-shard call) counted once, work x{S}",
+            "s_per_iter_extrapolated": s_per_build, "sample_s": ts, "overhead_s": ovh, "extrapolated": True}
 
 
 # ---------------------------------------------------------------------------------------------
 def run_reference(args):
-    """--impl reference: the oracle (plain C, OpenMP) timed on the host cores, rank 0 only."""
+    """--impl reference: the oracle (plain C, OpenMP) timed on the host cores, rank 0 only.  Each step is
+    one strided sample of canonical bra pairs (a different shard per step), sized and extrapolated exactly
+    as bench.py's cpu_baseline leg (per-call overhead measured on an empty shard and counted once)."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
@@ -196,38 +230,28 @@ def run_reference(args):
     D = mi.synthetic_density(n, mol.nelec // 2, seed=0)
     Q = oracle.schwarz(sh)
     total, nq = workload_flops(sh, Q, args.tau)
-    npair = sh.nshell * (sh.nshell + 1) // 2
-    # size one step at ~args.ref_step_s seconds of oracle work: pilot on 8 spread-out shards of 1/S0
-    # (one tiny shard is dominated by the per-call overhead and would overstate the build time), then
-    # a second pilot at the resulting size
-    S = max(2, min(npair, 20000))
-    t0 = time.perf_counter()
-    for i in range(8):
-        oracle.jk(sh, D, args.tau, (i * S) // 8 + 1, S, Q=Q)
-    est_total = max((time.perf_counter() - t0) / 8, 1e-4) * S
-    S = int(min(max(2, est_total / args.ref_step_s), npair))
-    t0 = time.perf_counter()
-    oracle.jk(sh, D, args.tau, S // 3, S, Q=Q)
-    est_total = max(time.perf_counter() - t0, 1e-4) * S
-    S = int(min(max(2, est_total / args.ref_step_s), npair))
-    times = []
+    S, ovh = oracle_sample_seconds(sh, D, args.tau, Q, args.ref_step_s)
+    S = max(S, 2)
+    builds, samples = [], []
     for i in range(args.warmup + args.steps):
-        shard = (7 * i + 1) % S
-        t0 = time.perf_counter()
-        oracle.jk(sh, D, args.tau, shard, S, Q=Q)
+        shard = (7 * i + S // 2) % S
+        ts, sb = oracle_sampled_build(sh, D, args.tau, Q, S, shard, ovh)
         if i >= args.warmup:
-            times.append(time.perf_counter() - t0)
-    s_per_build = float(np.mean(times)) * S
+            builds.append(sb)
+            samples.append(ts)
+    s_per_build = float(np.mean(builds))
     value = total / s_per_build / 1e12
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": s_per_build * 1e3, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": s_per_build * 1e3, "higher_is_better": True,
             "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "extrapolated": True, "sample_s_per_step": samples, "overhead_s": ovh,
             "config": {"workload": args.config, "basis": mi.basis_label(basis), "nbf": n, "tau": args.tau,
                        "quartets": nq, "gemm_flops_per_build": total},
             "s_per_iter": s_per_build,
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
                              "sample": f"each step: canonical bra pairs with index % {S} == shard (1/{S} of the "
-                                       f"build, shards vary per step), extrapolated x{S}"},
+                                       f"build, shards vary per step; {np.mean(samples):.1f} s measured per step), "
+                                       f"work x{S} + per-call overhead {ovh:.2f} s once (extrapolated)"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0

@@ -108,12 +108,15 @@ void mako_pairs_destroy(mako_pairs pairs);
  *         this shard that survive Q_ab Q_cd >= thresh.  Both come out exactly symmetric.
  *   thresh >= the pairs' screening threshold (smaller values are treated as equal to it).
  *   shard, nshards: 0 <= shard < nshards.  The canonical quartet tasks of every angular-momentum
- *         class are split into nshards contiguous ranges of equal modelled cost (primitive quartets,
- *         ket primitive pairs and quartets, weighted by the class's work per unit);
- *         shard `shard` takes its range.
+ *         class (in bra-Q-descending order) are cut into chunks of C consecutive tasks (C a multiple
+ *         of 4, about 256 chunks per shard); chunk j belongs to shard j mod nshards (interleaved, so
+ *         every shard samples the whole cost profile of the class).
  *         A pure function of (pairs, thresh, shard, nshards): summing J/K over all shards gives the
  *         nshards = 1 result up to FP64 summation order.
- *   cuda_stream: all work is enqueued on it (async).  J, K, D must not alias. */
+ *   cuda_stream: all work is enqueued on it (async).  J, K, D must not alias.  Builds on one pairs
+ *         handle are serialised: a build first waits (on cuda_stream) for the previous build of the
+ *         same handle, whatever stream that one was enqueued on (the task counters, the D block maxima
+ *         and the accumulate scratch are per-handle state). */
 mako_status mako_build_jk(mako_pairs pairs, const double* D, double thresh, double* J, double* K, int shard,
                           int nshards, void* cuda_stream);
 
@@ -128,6 +131,12 @@ mako_status mako_build_jk(mako_pairs pairs, const double* D, double thresh, doub
  * maxima on the device and SYNCHRONISES cuda_stream once (the task plan depends on max|D|);
  * otherwise identical to mako_build_jk (flags = 0 is exactly mako_build_jk). */
 #define MAKO_JK_DENSITY_SCREEN 1u
+/* flags |= MAKO_JK_ACCUMULATE: J and K are ACCUMULATED (J += J[D], K += K[D]) instead of overwritten.
+ * Used for incremental SCF builds on a density change (PAPER.md:L300 convergence-aware scheduling;
+ * SURVEY S8.f row 2): J[D_n] = J[D_{n-1}] + J[D_n - D_{n-1}] (J, K linear in D).  The build's own
+ * accumulators then live in a per-handle scratch of 2 nbf^2 doubles (allocated on first use), added
+ * into J/K by the final symmetrisation kernel.  Valid for mako_build_jk_ex and mako_build_jk_mixed. */
+#define MAKO_JK_ACCUMULATE 2u
 mako_status mako_build_jk_ex(mako_pairs pairs, const double* D, double thresh, unsigned flags, double* J, double* K,
                              int shard, int nshards, void* cuda_stream);
 
@@ -145,10 +154,16 @@ mako_status mako_build_jk_ex(mako_pairs pairs, const double* D, double thresh, u
  * with FP32 accumulation (L296 first stage) and digests into FP64 J/K (L296 second stage).  Classes
  * without a reduced-precision kernel (mako_class_reduced) run FP64 in both tiers.  Per-quartet error
  * budget: |d(ab|cd)| <= (2^-9 + (K1+K2) 2^-24) * sum|E~ R E~| (eri_quant.cuh).  thresh_fp64 > 0
- * (finite); thresh as in mako_build_jk_ex; flags: 0 or MAKO_JK_DENSITY_SCREEN.  SYNCHRONISES
+ * (finite); thresh as in mako_build_jk_ex; flags: MAKO_JK_DENSITY_SCREEN and/or MAKO_JK_ACCUMULATE.  SYNCHRONISES
  * cuda_stream once (max|D| decides the tier plan).  D, J, K as in mako_build_jk. */
 mako_status mako_build_jk_mixed(mako_pairs pairs, const double* D, double thresh, double thresh_fp64,
                                 unsigned flags, double* J, double* K, int shard, int nshards, void* cuda_stream);
+/* Density change of an incremental build: dD = D - D_prev (DEVICE nbf x nbf FP64,
+ * caller-owned; dD must not alias D or D_prev) and *dmax = max |dD| (HOST), which the caller's
+ * convergence-aware threshold schedule needs.  Enqueued on cuda_stream, then SYNCHRONISES it (dmax is
+ * returned).  A non-finite entry returns MAKO_ERR_INVALID (after writing dD). */
+mako_status mako_density_delta(mako_pairs pairs, const double* D, const double* D_prev, double* dD, double* dmax,
+                               void* cuda_stream);
 /* family[MAKO_NCLASS] (HOST): the kernel family that runs each class (S6): 0 lane-per-ket
  * register kernel, 1 ket-first DMMA kernel, 2 ket-first transposed, 3 slot-batched DMMA kernel,
  * 4 warp-per-quartet DMMA kernel.  For measurement reports. */

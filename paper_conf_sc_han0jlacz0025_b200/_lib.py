@@ -22,7 +22,8 @@ EXPORTS = ["mako_basis_create", "mako_basis_nbf", "mako_basis_nshell", "mako_bas
            "mako_shellpairs_screen", "mako_pairs_stats", "mako_pairs_flops", "mako_pairs_destroy", "mako_build_jk",
            "mako_build_jk_launches", "mako_eri_batch", "mako_boys", "mako_last_error", "mako_version",
            "mako_pairs_class_flops", "mako_profile_enable", "mako_profile_read", "mako_build_jk_ex",
-           "mako_build_jk_mixed", "mako_class_reduced", "mako_eri_batch_ex", "mako_class_family"]
+           "mako_build_jk_mixed", "mako_class_reduced", "mako_eri_batch_ex", "mako_class_family",
+           "mako_density_delta"]
 
 
 class MakoError(RuntimeError):
@@ -64,6 +65,7 @@ def load():
                              ctypes.c_int),
         "mako_build_jk_mixed": ([_vp, _vp, ctypes.c_double, ctypes.c_double, ctypes.c_uint, _vp, _vp, ctypes.c_int,
                                  ctypes.c_int, _vp], ctypes.c_int),
+        "mako_density_delta": ([_vp, _vp, _vp, _vp, _dp, _vp], ctypes.c_int),
         "mako_class_reduced": ([_ip], ctypes.c_int),
         "mako_class_family": ([_ip], ctypes.c_int),
         "mako_eri_batch_ex": ([_vp, ctypes.c_int, _ip, _vp, ctypes.c_size_t, ctypes.c_uint, _vp], ctypes.c_int),

@@ -280,6 +280,9 @@ extern "C" mako_status mako_basis_create(int natm, const int* Z, const double* x
         (st = upload(B->d_poff, B->poff)) || (st = upload(B->d_exps, B->exps)) || (st = upload(B->d_cn, B->cn)) ||
         (st = upload(B->d_sph, sph)) || (st = upload(B->d_boys, boys)))
       return st;
+    // pageable cudaMemcpy may return before its DMA lands; the pair builder runs on the caller's
+    // (possibly non-blocking) stream: finish the uploads here
+    if (cudaDeviceSynchronize() != cudaSuccess) return fail(MAKO_ERR_CUDA, "basis upload");
     *out = B.release();
     return MAKO_OK;
   } catch (const std::exception& e) {

@@ -27,6 +27,7 @@ bool lowp_xy();
 
 #ifdef MAKO_DEFINE_KERNELS
 #include <algorithm>
+#include <cstdlib>
 
 #include "eri_core.cuh"
 #include "eri_tpq.cuh"
@@ -48,6 +49,9 @@ constexpr bool has_lowp() {
   return !use_tpq(X, Y) && !use_kf<X, Y>() && !use_kf_swap<X, Y>() && !use_slab<X, Y>() && C::LA <= 3 &&
          C::LC <= 3 && C::NAB >= 9 && C::L >= 6;
 }
+
+template <int X, int Y>
+using JkCls = ClsXY<(use_jk_swap<X, Y>() ? Y : X), (use_jk_swap<X, Y>() ? X : Y)>;
 
 // warps per CTA of the warp-per-quartet kernels: 4, fewer when the per-warp SMEM of a class does
 // not fit (l = 4 classes: (gg|gg) runs 2 warps per CTA)
@@ -99,12 +103,8 @@ __device__ __forceinline__ void jk_body(const JKArgs& a) {
   double* V = Rbuf + C::W_R;
   double* jab = V + C::W_V;
   for (;;) {
-  unsigned long long grab = 0;
-  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
-  grab = __shfl_sync(0xffffffffu, grab, 0);
-  const long long tg0 = a.task_begin + (long long)grab;
-  if (tg0 >= a.task_end) break;
-  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  long long tg0, tg1;
+  if (!grab_tasks(a, lane, tg0, tg1)) break;
   int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;
@@ -184,12 +184,8 @@ __global__ void __launch_bounds__(CTA_THREADS) jk_kernel_q(JKArgs a) {
   double* jab = V + C::W_V;
   float* R32 = reinterpret_cast<float*>(Rbuf + C::WARP_DBL);
   for (;;) {
-  unsigned long long grab = 0;
-  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
-  grab = __shfl_sync(0xffffffffu, grab, 0);
-  const long long tg0 = a.task_begin + (long long)grab;
-  if (tg0 >= a.task_end) break;
-  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  long long tg0, tg1;
+  if (!grab_tasks(a, lane, tg0, tg1)) break;
   int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;
@@ -302,6 +298,11 @@ int jk_blocks_per_sm() {
       constexpr size_t ss = SlabCfg<X, Y>::SMEM;
       if (set_smem_attr<X, Y>((const void*)slab_jk_kernel<X, Y>, ss)) return 1;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, slab_jk_kernel<X, Y>, CTA_THREADS, ss);
+    } else if constexpr (use_jk_swap<X, Y>()) {
+      using CS = ClsXY<Y, X>;
+      constexpr size_t sms = cta_smem_bytes<CS>();
+      if (set_smem_attr<X, Y>((const void*)jk_kernel_ptr<Y, X>(), sms)) return 1;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel_ptr<Y, X>(), 32 * jk_warps<CS>(), sms);
     } else {
       if (set_smem_attr<X, Y>((const void*)jk_kernel_ptr<X, Y>(), smem)) return 1;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, jk_kernel_ptr<X, Y>(), 32 * jk_warps<C>(), smem);
@@ -315,14 +316,14 @@ template <int X, int Y>
 mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   using C = ClsXY<X, Y>;
   constexpr size_t smem = cta_smem_bytes<C>();
-  const long long ntask = a.task_end - a.task_begin;
+  const long long ntask = a.ntask_local;
   if (ntask <= 0) return MAKO_OK;
   int dev = 0, nsm = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   const int bps = jk_blocks_per_sm<X, Y>();
   constexpr int WPC = (use_kf_swap<X, Y>() || use_kf<X, Y>() || use_tpq(X, Y) || use_slab<X, Y>()) ? CTA_WARPS
-                                                                                                 : jk_warps<C>();
+                                                                                                 : jk_warps<JkCls<X, Y>>();
   long long want = (ntask + WPC - 1) / WPC;
   long long cap = (long long)nsm * bps / (a.grid_div > 1 ? a.grid_div : 1);
   if (cap < nsm) cap = nsm;
@@ -332,20 +333,22 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
   const cudaStream_t cs = (cudaStream_t)stream;
   if constexpr (has_lowp<X, Y>()) {
     if (a.lowp) {
-      constexpr size_t sq = cta_smem_bytes_q<C>();
+      constexpr int XQ = use_jk_swap<X, Y>() ? Y : X, YQ = use_jk_swap<X, Y>() ? X : Y;
+      using CQ = ClsXY<XQ, YQ>;
+      constexpr size_t sq = cta_smem_bytes_q<CQ>();
       // the TF32 tier's own occupancy (its SMEM is larger by the TF32 R rows)
       static int bq = -1;
       if (bq < 0) {
-        if (set_smem_attr<X, Y>((const void*)jk_kernel_q<X, Y>, sq) ||
-            set_smem_attr<X, Y>((const void*)jk_kernel_q<X, Y, true>, sq))
+        if (set_smem_attr<X, Y>((const void*)jk_kernel_q<XQ, YQ>, sq) ||
+            set_smem_attr<X, Y>((const void*)jk_kernel_q<XQ, YQ, true>, sq))
           return MAKO_ERR_CUDA;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bq, jk_kernel_q<X, Y>, 32 * q_warps<C>(), sq);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bq, jk_kernel_q<XQ, YQ>, 32 * q_warps<CQ>(), sq);
         if (bq < 1) bq = 1;
       }
-      constexpr int QW = q_warps<C>();
+      constexpr int QW = q_warps<CQ>();
       const long long gq = std::min<long long>((ntask + QW - 1) / QW, std::max<long long>((long long)nsm * bq, nsm));
-      if (a.dsh) jk_kernel_q<X, Y, true><<<(int)gq, 32 * QW, sq, cs>>>(a);
-      else jk_kernel_q<X, Y><<<(int)gq, 32 * QW, sq, cs>>>(a);
+      if (a.dsh) jk_kernel_q<XQ, YQ, true><<<(int)gq, 32 * QW, sq, cs>>>(a);
+      else jk_kernel_q<XQ, YQ><<<(int)gq, 32 * QW, sq, cs>>>(a);
       cudaError_t e = cudaGetLastError();
       if (e != cudaSuccess) return fail(MAKO_ERR_CUDA, std::string("jk_kernel_q launch: ") + cudaGetErrorString(e));
       if (nlaunch) ++*nlaunch;
@@ -367,14 +370,35 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
       kf_jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, cs>>>(a);
     }
   } else if constexpr (use_tpq(X, Y)) {
-    if (a.dsh) tpq_jk_kernel<X, Y, true><<<grid, CTA_THREADS, 0, cs>>>(a);
-    else tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, cs>>>(a);
+    // strip digestion when the bra unit's K rows fit in shared memory (eri_tpq.cuh)
+    static const bool no_strip = std::getenv("MAKO_NO_STRIP") != nullptr;  // A/B experiments only
+    const size_t ss = tpq_strip_smem<X, Y>(a.nbf, a.nshell);
+    if (!no_strip && a.unit_off && ss <= SMEM_CTA_MAX) {
+      const void* fn = a.dsh ? (const void*)tpq_strip_kernel<X, Y, true> : (const void*)tpq_strip_kernel<X, Y>;
+      if (set_smem_attr<X, Y>(fn, ss)) return MAKO_ERR_CUDA;
+      int nb = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, tpq_strip_kernel<X, Y>, 32 * TPQ_STRIP_WARPS, ss);
+      const long long gs = std::min<long long>((long long)nsm * std::max(nb, 1), a.nunit);
+      if (a.dsh) tpq_strip_kernel<X, Y, true><<<(int)std::max<long long>(gs, 1), 32 * TPQ_STRIP_WARPS, ss, cs>>>(a);
+      else tpq_strip_kernel<X, Y><<<(int)std::max<long long>(gs, 1), 32 * TPQ_STRIP_WARPS, ss, cs>>>(a);
+    } else {
+      if (a.dsh) tpq_jk_kernel<X, Y, true><<<grid, CTA_THREADS, 0, cs>>>(a);
+      else tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, cs>>>(a);
+    }
   } else if constexpr (use_slab<X, Y>()) {
     if (a.dsh) {
       if (set_smem_attr<X, Y>((const void*)slab_jk_kernel<X, Y, true>, SlabCfg<X, Y>::SMEM)) return MAKO_ERR_CUDA;
       slab_jk_kernel<X, Y, true><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, cs>>>(a);
     } else {
       slab_jk_kernel<X, Y><<<grid, CTA_THREADS, SlabCfg<X, Y>::SMEM, cs>>>(a);
+    }
+  } else if constexpr (use_jk_swap<X, Y>()) {
+    constexpr size_t sms = cta_smem_bytes<ClsXY<Y, X>>();
+    if (a.dsh) {
+      if (set_smem_attr<X, Y>((const void*)jk_kernel_ptr<Y, X, true>(), sms)) return MAKO_ERR_CUDA;
+      jk_kernel_ptr<Y, X, true>()<<<grid, 32 * WPC, sms, cs>>>(a);
+    } else {
+      jk_kernel_ptr<Y, X>()<<<grid, 32 * WPC, sms, cs>>>(a);
     }
   } else {
     if (a.dsh) {
@@ -429,7 +453,7 @@ int task_kets_xy() {
 }
 template <int X, int Y>
 bool swap_xy() {
-  return use_kf_swap<X, Y>();
+  return use_kf_swap<X, Y>() || use_jk_swap<X, Y>();
 }
 template <int X, int Y>
 bool lowp_xy() {

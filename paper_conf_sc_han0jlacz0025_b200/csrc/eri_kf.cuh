@@ -93,12 +93,8 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
   for (int i = lane; i < K::WARP_DBL; i += 32) Ws[i] = 0.0;  // padding rows/cols stay zero forever
   __syncwarp();
   for (;;) {
-  unsigned long long grab = 0;
-  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
-  grab = __shfl_sync(0xffffffffu, grab, 0);
-  const long long tg0 = a.task_begin + (long long)grab;
-  if (tg0 >= a.task_end) break;
-  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  long long tg0, tg1;
+  if (!grab_tasks(a, lane, tg0, tg1)) break;
   int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;

@@ -17,6 +17,7 @@
 
 #include "eri_core.cuh"
 #include "eri_tpq.cuh"
+#include "eri_kf.cuh"
 
 namespace mako {
 
@@ -53,6 +54,15 @@ constexpr bool use_slab() {
   return !use_tpq(X, Y) && SlabCfg<X, Y>::OK && in_list(kSlabPick, X * 100 + Y);
 }
 
+// warp-per-quartet class run transposed: task pairs from the ket bucket Y, kets from X (jk_kernel<Y, X>
+// evaluates (cd|ab) = (ab|cd) and digests it with the same six updates); its reduced tier runs
+// jk_kernel_q<Y, X> likewise
+template <int X, int Y>
+constexpr bool use_jk_swap() {
+  return X != Y && !use_tpq(X, Y) && !use_kf<X, Y>() && !use_kf_swap<X, Y>() && !use_slab<X, Y>() &&
+         in_list(kJkSwapPick, X * 100 + Y);
+}
+
 template <int X, int Y, bool DW = false>
 __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
   using C = ClsXY<X, Y>;
@@ -84,12 +94,8 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
   for (int i = lane; i < S::W_R; i += 32) Rs[i] = 0.0;  // unused slots must stay finite
   __syncthreads();
   for (;;) {
-  unsigned long long grab = 0;
-  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
-  grab = __shfl_sync(0xffffffffu, grab, 0);
-  const long long tg0 = a.task_begin + (long long)grab;
-  if (tg0 >= a.task_end) break;
-  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
+  long long tg0, tg1;
+  if (!grab_tasks(a, lane, tg0, tg1)) break;
   int U = find_entry(a, tg0);
   for (long long task = tg0; task < tg1; ++task) {
     while (__ldg(a.task_off + U + 1) <= task) ++U;

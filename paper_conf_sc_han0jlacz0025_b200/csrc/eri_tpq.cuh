@@ -124,10 +124,19 @@ constexpr bool tpq_wacc() {
   return nH(C::L) + C::NAB * C::NCD + C::NHAB * C::NCD + C::NHCD * C::NCD <= 110;
 }
 
-#ifndef MAKO_TASK_GRAB
-#define MAKO_TASK_GRAB 4
-#endif
-constexpr int TASK_GRAB = MAKO_TASK_GRAB;  // tasks taken per counter increment (one entry lookup per grab)
+// One grab of the persistent task loop: lane 0 takes TASK_GRAB local tasks from the class counter;
+// returns false when the shard's tasks are exhausted, else the global task range [tg0, tg1) (never
+// crosses a shard chunk: chunk sizes are multiples of TASK_GRAB and grabs start at multiples of it).
+__device__ __forceinline__ bool grab_tasks(const JKArgs& a, int lane, long long& tg0, long long& tg1) {
+  unsigned long long grab = 0;
+  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
+  grab = __shfl_sync(0xffffffffu, grab, 0);
+  const long long l0 = (long long)grab;
+  if (l0 >= a.ntask_local) return false;
+  tg0 = a.nshards == 1 ? l0 : shard_task(l0, a.shard, a.nshards, a.chunk);
+  tg1 = min(tg0 + TASK_GRAB, a.ntask);
+  return true;
+}
 
 // density-weighted screening of quartet (sa sb|sc sd) with Schwarz product qq (reading R17)
 template <bool DW>
@@ -148,32 +157,27 @@ __device__ __forceinline__ int find_entry(const JKArgs& a, long long task) {
   return U;
 }
 
-// Persistent lane-per-ket kernel (JKArgs.KT must be 32).
-#ifdef MAKO_TPQ_MINB
-#define MAKO_TPQ_BOUNDS __launch_bounds__(128, MAKO_TPQ_MINB)
-#else
-#define MAKO_TPQ_BOUNDS __launch_bounds__(128)
-#endif
-template <int X, int Y, bool DW = false>
-__global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
+// K-row strip of a bra unit in shared memory (strip digestion, S6): rows 0..NA-1 hold
+// K[oa + i][*], rows NA..NA+NB-1 hold K[ob + j][*], full nbf columns; J_ab partial sums behind them;
+// a bitmap of the ket shells whose columns were touched.  Flushed to global J/K once per bra unit.
+struct Strip {
+  double* K;          // [(NA + NB) * nbf]
+  double* Jab;        // [NAB]
+  unsigned* touched;  // [(nshell + 31) / 32]
+};
+
+// shared-memory double add (sm_100a has no native f64 shared atomic: CAS loop, rarely contended here)
+__device__ __forceinline__ void sh_add(double* p, double v) { atomicAdd(p, v); }
+
+// One lane-per-ket task: bra pair P, kets [r0, r1) (<= 32, lane i takes ket r0 + i).  Boys, R, the
+// ket-first contraction and digestion all in registers.  STRIP: the K_ac/K_ad/K_bc/K_bd updates and
+// J_ab go to the CTA's shared K-row strip of bra P instead of global FP64 atomics (J_cd stays global).
+template <int X, int Y, bool DW, bool STRIP>
+__device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1, int lane, const Strip& st) {
   using C = ClsXY<X, Y>;
   constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
   constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND;
   constexpr bool WACC = tpq_wacc<C>();
-  const int lane = threadIdx.x & 31;
-  for (;;) {
-  unsigned long long grab = 0;
-  if (lane == 0) grab = atomicAdd(a.counter, (unsigned long long)TASK_GRAB);
-  grab = __shfl_sync(0xffffffffu, grab, 0);
-  const long long tg0 = a.task_begin + (long long)grab;
-  if (tg0 >= a.task_end) break;
-  const long long tg1 = min(tg0 + TASK_GRAB, a.task_end);
-  int U = find_entry(a, tg0);
-  for (long long task = tg0; task < tg1; ++task) {
-    while (__ldg(a.task_off + U + 1) <= task) ++U;
-    const int P = __ldg(a.ent_P + U);
-    const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * 32;
-    const int r1 = min(r0 + 32, __ldg(a.kend + U));
     const int R = r0 + lane;
     const double QP = __ldg(a.bra.Q + P);
     const double QQ = QP * __ldg(a.ket.Q + min(R, r1 - 1));
@@ -288,9 +292,12 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
       s *= deg;
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-      if (lane == 0) atomicAdd(a.J + (oa + i / NB) * n + ob + i % NB, 2.0 * s);
+      if (lane == 0) {
+        if constexpr (STRIP) sh_add(st.Jab + i, 2.0 * s);
+        else atomicAdd(a.J + (oa + i / NB) * n + ob + i % NB, 2.0 * s);
+      }
     }
-    if (!active) continue;
+    if (!active) return;
     // J_cd
 #pragma unroll
     for (int k = 0; k < NC; ++k)
@@ -301,7 +308,12 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
         for (int ij = 0; ij < NAB; ++ij) s = fma(V[ij][k * ND + l], __ldg(Dm + (oa + ij / NB) * n + ob + ij % NB), s);
         atomicAdd(a.J + (oc + k) * n + od + l, 2.0 * deg * s);
       }
+    if constexpr (STRIP) {
+      atomicOr(st.touched + (sc >> 5), 1u << (sc & 31));
+      atomicOr(st.touched + (sd >> 5), 1u << (sd & 31));
+    }
     // K_ac += v D_bd ; K_ad += v D_bc ; K_bc += v D_ad ; K_bd += v D_ac
+    // (strip: row i of shell a is strip row i, row j of shell b is strip row NA + j, column = AO index)
 #pragma unroll
     for (int i = 0; i < NA; ++i)
 #pragma unroll
@@ -311,7 +323,8 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
         for (int j = 0; j < NB; ++j)
 #pragma unroll
           for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (ob + j) * n + od + l), s);
-        atomicAdd(a.K + (oa + i) * n + oc + k, deg * s);
+        if constexpr (STRIP) sh_add(st.K + i * n + oc + k, deg * s);
+        else atomicAdd(a.K + (oa + i) * n + oc + k, deg * s);
       }
 #pragma unroll
     for (int i = 0; i < NA; ++i)
@@ -322,7 +335,8 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
         for (int j = 0; j < NB; ++j)
 #pragma unroll
           for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (ob + j) * n + oc + k), s);
-        atomicAdd(a.K + (oa + i) * n + od + l, deg * s);
+        if constexpr (STRIP) sh_add(st.K + i * n + od + l, deg * s);
+        else atomicAdd(a.K + (oa + i) * n + od + l, deg * s);
       }
 #pragma unroll
     for (int j = 0; j < NB; ++j)
@@ -333,7 +347,8 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
         for (int i = 0; i < NA; ++i)
 #pragma unroll
           for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (oa + i) * n + od + l), s);
-        atomicAdd(a.K + (ob + j) * n + oc + k, deg * s);
+        if constexpr (STRIP) sh_add(st.K + (NA + j) * n + oc + k, deg * s);
+        else atomicAdd(a.K + (ob + j) * n + oc + k, deg * s);
       }
 #pragma unroll
     for (int j = 0; j < NB; ++j)
@@ -344,9 +359,109 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
         for (int i = 0; i < NA; ++i)
 #pragma unroll
           for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Dm + (oa + i) * n + oc + k), s);
-        atomicAdd(a.K + (ob + j) * n + od + l, deg * s);
+        if constexpr (STRIP) sh_add(st.K + (NA + j) * n + od + l, deg * s);
+        else atomicAdd(a.K + (ob + j) * n + od + l, deg * s);
       }
+}
+
+// Persistent lane-per-ket kernel (JKArgs.KT must be 32).
+#ifdef MAKO_TPQ_MINB
+#define MAKO_TPQ_BOUNDS __launch_bounds__(128, MAKO_TPQ_MINB)
+#else
+#define MAKO_TPQ_BOUNDS __launch_bounds__(128)
+#endif
+template <int X, int Y, bool DW = false>
+__global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
+  const int lane = threadIdx.x & 31;
+  for (;;) {
+  long long tg0, tg1;
+  if (!grab_tasks(a, lane, tg0, tg1)) break;
+  int U = find_entry(a, tg0);
+  for (long long task = tg0; task < tg1; ++task) {
+    while (__ldg(a.task_off + U + 1) <= task) ++U;
+    const int P = __ldg(a.ent_P + U);
+    const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * 32;
+    const int r1 = min(r0 + 32, __ldg(a.kend + U));
+    tpq_task<X, Y, DW, false>(a, P, r0, r1, lane, Strip{});
   }
+  }
+}
+
+// Strip-digestion variant (S6, "K-row strips"): a CTA takes a whole bra unit (every task of
+// one bra pair P, all ket K-groups) from the class's unit counter; its warps share the unit's tasks and
+// accumulate K rows of shells a and b (all nbf columns) and J_ab in shared memory; the touched ket-shell
+// columns are flushed to global memory with one FP64 atomic per element once per unit.  Per quartet
+// the global atomics drop from NCD + (NA+NB)(NC+ND) to NCD (J_cd).  Used when the strip fits in shared
+// memory ((NA+NB) nbf doubles); a unit's tasks outside this launch's shard are skipped.
+constexpr int TPQ_STRIP_WARPS = 8;
+template <int X, int Y>
+__host__ __device__ constexpr size_t tpq_strip_smem(int nbf, int nshell) {
+  using C = ClsXY<X, Y>;
+  return sizeof(double) * ((size_t)(C::NA + C::NB) * nbf + C::NAB) + sizeof(unsigned) * (size_t)((nshell + 31) / 32 + 1);
+}
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(32 * TPQ_STRIP_WARPS) tpq_strip_kernel(JKArgs a) {
+  using C = ClsXY<X, Y>;
+  constexpr int NA = C::NA, NB = C::NB, NAB = C::NAB;
+  extern __shared__ __align__(16) double strip_smem[];
+  __shared__ int s_unit;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nbf = a.nbf, nw = (a.nshell + 31) / 32;
+  Strip st;
+  st.K = strip_smem;
+  st.Jab = strip_smem + (size_t)(NA + NB) * nbf;
+  st.touched = reinterpret_cast<unsigned*>(st.Jab + NAB);
+  for (int i = threadIdx.x; i < (NA + NB) * nbf + NAB; i += blockDim.x) strip_smem[i] = 0.0;
+  for (int i = threadIdx.x; i < nw; i += blockDim.x) st.touched[i] = 0u;
+  __syncthreads();
+  for (;;) {
+    if (threadIdx.x == 0) s_unit = (int)atomicAdd(a.counter, 1ull);
+    __syncthreads();
+    const int u = s_unit;
+    if (u >= a.nunit) break;
+    const long long t0 = __ldg(a.unit_off + u), t1 = __ldg(a.unit_off + u + 1);
+    const int P = __ldg(a.unit_P + u);
+    // the unit's tasks (this shard's part), round-robin over the warps
+    int U = -1;
+    for (long long task = t0 + warp; task < t1; task += TPQ_STRIP_WARPS) {
+      if (a.nshards > 1 && (task / a.chunk) % a.nshards != a.shard) continue;
+      if (U < 0) U = find_entry(a, task);
+      while (__ldg(a.task_off + U + 1) <= task) ++U;
+      const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * 32;
+      const int r1 = min(r0 + 32, __ldg(a.kend + U));
+      tpq_task<X, Y, DW, true>(a, P, r0, r1, lane, st);
+    }
+    __syncthreads();
+    // flush: J_ab, then the touched columns of the K rows of a and b (zeroing them for the next unit)
+    const int sa = __ldg(a.bra.shA + P), sb = __ldg(a.bra.shB + P);
+    const int oa = __ldg(a.ao + sa), ob = __ldg(a.ao + sb);
+    for (int i = threadIdx.x; i < NAB; i += blockDim.x) {
+      const double v = st.Jab[i];
+      if (v != 0.0) {
+        atomicAdd(a.J + (size_t)(oa + i / NB) * nbf + ob + i % NB, v);
+        st.Jab[i] = 0.0;
+      }
+    }
+    for (int w = warp; w < nw; w += TPQ_STRIP_WARPS) {
+      unsigned bits = st.touched[w];
+      while (bits) {
+        const int x = 32 * w + __ffs(bits) - 1;
+        bits &= bits - 1;
+        const int ox = __ldg(a.ao + x), nx = 2 * __ldg(a.shl + x) + 1;
+        for (int e = lane; e < (NA + NB) * nx; e += 32) {
+          const int row = e / nx, col = ox + e % nx;
+          double* p = st.K + (size_t)row * nbf + col;
+          const double v = *p;
+          if (v != 0.0) {
+            atomicAdd(a.K + (size_t)(row < NA ? oa + row : ob + row - NA) * nbf + col, v);
+            *p = 0.0;
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) st.touched[w] = 0u;
+    }
+    __syncthreads();
   }
 }
 

@@ -63,10 +63,11 @@ static bool class_swap(int X, int Y) {
 }
 
 // kernel family of a class (include/mako.h mako_class_family): 0 lane-per-ket (tpq), 1 ket-first (kf),
-// 2 ket-first transposed, 3 slot-batched (slab), 4 warp-per-quartet (jk)
+// 2 ket-first transposed, 3 slot-batched (slab), 4 warp-per-quartet (jk), 5 warp-per-quartet transposed
 template <int X, int Y>
 static int family_xy() {
   if constexpr (use_kf_swap<X, Y>()) return 2;
+  else if constexpr (use_jk_swap<X, Y>()) return 5;
   else if constexpr (use_kf<X, Y>()) return 1;
   else if constexpr (use_tpq(X, Y)) return 0;
   else if constexpr (use_slab<X, Y>()) return 3;
@@ -101,6 +102,17 @@ static mako_status upload(DevBuf& d, const std::vector<T>& h) {
   return MAKO_OK;
 }
 
+// stream-ordered upload (the kernels reading the buffer are launched on the same stream afterwards;
+// a pageable source is staged before cudaMemcpyAsync returns, so `h` may die right after)
+template <class T>
+static mako_status upload_async(DevBuf& d, const std::vector<T>& h, cudaStream_t s) {
+  mako_status st = d.alloc(h.size() * sizeof(T));
+  if (st) return st;
+  if (!h.empty())
+    return cuda_check(cudaMemcpyAsync(d.p, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice, s), "upload");
+  return MAKO_OK;
+}
+
 // number of kets R in [lo, hi) of bucket Y (Q-sorted desc within the segment) with QP * Q[R] >= thresh
 static int prefix_count(const std::vector<double>& QY, int lo0, int hi0, double QP, double thresh) {
   int lo = lo0, hi = hi0;
@@ -116,20 +128,10 @@ static int prefix_count(const std::vector<double>& QY, int lo0, int hi0, double 
 static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const PairBucket& by, bool same, double lo,
                                     double hi) {
   const int nbra = bx.n(), G = NKGROUP;
-  // shard-balance cost model of one quartet of this class (FLOP-like units): per primitive
-  // quartet the Boys seed + R recursion + GEMM1 row, per ket primitive pair GEMM2, per quartet the
-  // digestion and task overhead.  Measured: primitive quartets alone left shard 0 (many K = 1 bras)
-  // 25 % above the mean on the valinomycin build.
-  const int la = bx.la, lb = bx.lb, lc = by.la, ld = by.lb, L = la + lb + lc + ld;
-  const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
-  const double cA = 2.0 * nab * nH(la + lb) * nH(lc + ld) + 4.0 * nH(L) * (L + 1) + 60.0;
-  const double cB = 2.0 * nab * nH(lc + ld) * ncd;
-  const double cC = 12.0 * nab * ncd + 200.0;
   c.ent_P.clear();
   c.kbeg.clear();
   c.kend.clear();
   c.task_off.assign(1, 0);
-  c.cost_cum.assign(1, 0.0);
   c.nquartet = 0;
   for (int p = 0; p < nbra; ++p)
     for (int g = 0; g < G; ++g) {
@@ -147,10 +149,16 @@ static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const Pa
       c.kend.push_back(s0 + nk);
       c.nquartet += nk - nh;
       c.task_off.push_back(c.task_off.back() + (nk - nh + c.KT - 1) / c.KT);
-      const double kab = bx.poff[p + 1] - bx.poff[p], skcd = by.poff[s0 + nk] - by.poff[s0 + nh];
-      c.cost_cum.push_back(c.cost_cum.back() + kab * skcd * cA + skcd * cB + (nk - nh) * cC);
     }
   c.ntask = c.task_off.back();
+  c.unit_off.clear();
+  c.unit_P.clear();
+  for (size_t u = 0; u < c.ent_P.size(); ++u)
+    if (u == 0 || c.ent_P[u] != c.ent_P[u - 1]) {
+      c.unit_off.push_back(c.task_off[u]);
+      c.unit_P.push_back(c.ent_P[u]);
+    }
+  c.unit_off.push_back(c.ntask);
   c.usamp.assign((size_t)(c.ntask >> TASK_SAMPLE_SHIFT) + 1, 0);
   for (size_t u = 0, k = 0; k < c.usamp.size(); ++k) {
     const long long t = (long long)k << TASK_SAMPLE_SHIFT;
@@ -160,27 +168,20 @@ static mako_status build_class_plan(ClassPlan& c, const PairBucket& bx, const Pa
   mako_status st;
   if (c.ntask > 0 && ((st = upload(c.d_kbeg, c.kbeg)) || (st = upload(c.d_kend, c.kend)) ||
                       (st = upload(c.d_task_off, c.task_off)) || (st = upload(c.d_ent_P, c.ent_P)) ||
-                      (st = upload(c.d_usamp, c.usamp))))
+                      (st = upload(c.d_usamp, c.usamp)) || (st = upload(c.d_unit_off, c.unit_off)) ||
+                      (st = upload(c.d_unit_P, c.unit_P))))
     return st;
   return MAKO_OK;
 }
 
-// Task index of the cut between shard s-1 and shard s of n (s = 0..n) in class plan c:
-// contiguous ranges of EQUAL COST (the cost model of build_class_plan), cut inside an entry in
-// proportion to its tasks.  A pure function of the plan, monotone in s.
-static long long shard_cut(const ClassPlan& c, int s, int n) {
-  if (s <= 0 || c.ntask == 0) return 0;
-  if (s >= n) return c.ntask;
-  const double total = c.cost_cum.back();
-  if (!(total > 0)) return c.ntask * s / n;
-  const double target = total * s / n;
-  size_t u = std::upper_bound(c.cost_cum.begin(), c.cost_cum.end(), target) - c.cost_cum.begin();
-  u = u == 0 ? 0 : u - 1;
-  if (u + 1 >= c.cost_cum.size()) return c.ntask;
-  const double w = c.cost_cum[u + 1] - c.cost_cum[u];
-  const long long nt = c.task_off[u + 1] - c.task_off[u];
-  const long long k = w > 0 ? std::llround((target - c.cost_cum[u]) / w * (double)nt) : 0;
-  return c.task_off[u] + std::min(std::max(k, 0LL), nt);
+// Global task ranges [t0, t1) of shard s of n in class plan c (the interleaved chunks of shard_chunk /
+// shard_task, mako_internal.h), in increasing order.
+template <class F>
+static void for_shard_ranges(const ClassPlan& c, int s, int n, F&& f) {
+  if (c.ntask == 0) return;
+  if (n == 1) { f(0LL, c.ntask); return; }
+  const long long C = shard_chunk(c.ntask, n);
+  for (long long j = s; j * C < c.ntask; j += n) f(j * C, std::min((j + 1) * C, c.ntask));
 }
 
 constexpr int KT_JK = 4;
@@ -188,11 +189,12 @@ constexpr int KT_JK = 4;
 // Plan for Schwarz threshold `thresh`; with tier > thresh (reduced-precision build)
 // the quartets of classes that have a TF32-tier kernel are split: Q_ab Q_cd >= tier into cls (FP64),
 // thresh <= Q_ab Q_cd < tier into cls_lo (TF32).  tier = 0: one FP64 tier.
-static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0) {
+static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0, int nshards = 1) {
   if (!(tier > thresh)) tier = 0.0;
-  if (P->plan.thresh == thresh && P->plan.tier == tier && !P->plan.cls.empty()) return MAKO_OK;
+  if (P->plan.thresh == thresh && P->plan.tier == tier && P->plan.nshards == nshards && !P->plan.cls.empty())
+    return MAKO_OK;
   for (auto& sp : P->plan_cache)
-    if (sp.thresh == thresh && sp.tier == tier && !sp.cls.empty()) {
+    if (sp.thresh == thresh && sp.tier == tier && sp.nshards == nshards && !sp.cls.empty()) {
       std::swap(P->plan, sp);
       return MAKO_OK;
     }
@@ -207,6 +209,11 @@ static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0) {
   pl.cls_lo.resize(NCL);
   pl.KT = 16;
   const double inf = std::numeric_limits<double>::infinity();
+  if (P->nsm <= 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&P->nsm, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || P->nsm <= 0) P->nsm = 148;
+  }
   for (int X = 0; X < NBUCKET; ++X)
     for (int Y = 0; Y <= X; ++Y) {
       const int ci = class_index(X, Y);
@@ -219,11 +226,11 @@ static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0) {
         // warp-per-quartet classes: 4 kets per task (measured on the bench workload, tools/exp/kt.sh:
         // family time 5.60 / 5.52 / 5.47 / 5.45 s at KT = 32 / 16 / 8 / 4; the slot-batched kernel
         // batches ket primitives across the kets of a task and keeps 16)
-        if (class_family(X, Y) == 4) c.KT = KT_JK;
+        if (class_family(X, Y) == 4 || class_family(X, Y) == 5) c.KT = KT_JK;
         {  // experiments only (tools/exp): MAKO_KT_EXP overrides the base task length of the runtime-KT families
           static const int kt_exp = std::getenv("MAKO_KT_EXP") ? std::atoi(std::getenv("MAKO_KT_EXP")) : 0;
           const int f = class_family(X, Y);
-          if (kt_exp > 0 && (f == 3 || f == 4)) c.KT = kt_exp;
+          if (kt_exp > 0 && (f == 3 || f == 4 || f == 5)) c.KT = kt_exp;
         }
         c.swap = class_swap(X, Y);
         c.TB = c.swap ? Y : X;
@@ -233,19 +240,23 @@ static mako_status ensure_plan(mako_pairs P, double thresh, double tier = 0.0) {
         if (st) return st;
         // warp-per-quartet and slot-batched classes (runtime KT) with few quartets (contracted or small
         // high-l workloads, e.g. the paper's E1 microbenchmark): shorter tasks so
-        // that the 148 SMs see at least ~32 grabs (TASK_GRAB tasks each) per SM instead of a few
-        // long-running warps
-        const long long want = (long long)TASK_GRAB * 148 * 32;
+        // that the SMs see at least ~32 grabs (TASK_GRAB tasks each) per SM instead of a few
+        // long-running warps; with nshards GPUs each one sees 1/nshards of the class
+        const long long want = (long long)TASK_GRAB * P->nsm * 32;
         const int fam = class_family(X, Y);
-        if ((fam == 4 || fam == 3) && c.nquartet > 0 && c.nquartet / c.KT < want) {
-          c.KT = (int)std::max<long long>(1, c.nquartet / want);
+        const long long nq_shard = c.nquartet / nshards;
+        if ((fam == 4 || fam == 3 || fam == 5) && nq_shard > 0 && nq_shard / c.KT < want) {
+          c.KT = (int)std::max<long long>(1, nq_shard / want);
           if ((st = build_class_plan(c, P->set.b[c.TB], P->set.b[c.LB], X == Y, lo, hi))) return st;
         }
       }
     }
   pl.thresh = thresh;
   pl.tier = tier;
-  return MAKO_OK;
+  pl.nshards = nshards;
+  // the plan arrays were uploaded with pageable cudaMemcpy (legacy stream); the kernels that read them
+  // run on non-blocking streams: wait for the DMA to land before any launch
+  return cuda_check(cudaDeviceSynchronize(), "plan upload");
 }
 
 // J = Jacc + Jacc^T, K = Kacc + Kacc^T (in place)
@@ -261,6 +272,36 @@ __global__ void symmetrize_kernel(double* __restrict__ J, double* __restrict__ K
   }
 }
 
+// accumulate mode (MAKO_JK_ACCUMULATE): J += Jacc + Jacc^T, K += Kacc + Kacc^T
+__global__ void symmetrize_add_kernel(const double* __restrict__ Ja, const double* __restrict__ Ka,
+                                      double* __restrict__ J, double* __restrict__ K, int n) {
+  const long long total = (long long)n * n;
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < total; x += (long long)gridDim.x * blockDim.x) {
+    const int i = (int)(x / n), j = (int)(x % n);
+    const size_t a = (size_t)i * n + j, b = (size_t)j * n + i;
+    J[a] += Ja[a] + Ja[b];
+    K[a] += Ka[a] + Ka[b];
+  }
+}
+
+// dD = D - Dprev and max |dD| (NaN-propagating, as dsh_kernel)
+__global__ void delta_kernel(const double* __restrict__ D, const double* __restrict__ Dp, double* __restrict__ dD,
+                             long long total, unsigned long long* __restrict__ dmax) {
+  double gm = 0.0;
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < total; x += (long long)gridDim.x * blockDim.x) {
+    const double v = D[x] - Dp[x];
+    dD[x] = v;
+    const double a = fabs(v);
+    gm = (a > gm || a != a) ? a : gm;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const double y = __shfl_xor_sync(0xffffffffu, gm, o);
+    gm = (y > gm || y != y) ? y : gm;
+  }
+  if ((threadIdx.x & 31) == 0) atomicMax(dmax, (unsigned long long)__double_as_longlong(gm));
+}
+
 // density screening: dsh[sa][sb] = max |D| over the (sa, sb) block (rounded up to float); dmax = max |D|
 __global__ void dsh_kernel(const double* __restrict__ D, int nbf, int nshell, const int* __restrict__ ao,
                            const int* __restrict__ l, float* __restrict__ dsh, unsigned long long* __restrict__ dmax) {
@@ -269,15 +310,23 @@ __global__ void dsh_kernel(const double* __restrict__ D, int nbf, int nshell, co
   for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < n2; x += (long long)gridDim.x * blockDim.x) {
     const int sa = (int)(x / nshell), sb = (int)(x % nshell);
     const int oa = ao[sa], ob = ao[sb], na = 2 * l[sa] + 1, nb = 2 * l[sb] + 1;
+    // NaN-propagating maxima (fmax drops NaN): a NaN anywhere in D makes dmax NaN and fails the build
     double m = 0.0;
     for (int i = 0; i < na; ++i)
-      for (int j = 0; j < nb; ++j) m = fmax(m, fabs(D[(size_t)(oa + i) * nbf + ob + j]));
+      for (int j = 0; j < nb; ++j) {
+        const double v = fabs(D[(size_t)(oa + i) * nbf + ob + j]);
+        m = (v > m || v != v) ? v : m;
+      }
     dsh[x] = __double2float_ru(m);
-    gm = fmax(gm, m);
+    gm = (m > gm || m != m) ? m : gm;
   }
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) gm = fmax(gm, __shfl_xor_sync(0xffffffffu, gm, o));
-  if ((threadIdx.x & 31) == 0) atomicMax(dmax, (unsigned long long)__double_as_longlong(gm));  // gm >= 0
+  for (int o = 16; o > 0; o >>= 1) {
+    const double y = __shfl_xor_sync(0xffffffffu, gm, o);
+    gm = (y > gm || y != y) ? y : gm;
+  }
+  // gm >= 0 or +NaN: as unsigned bit patterns these order like the values, NaN above +inf
+  if ((threadIdx.x & 31) == 0) atomicMax(dmax, (unsigned long long)__double_as_longlong(gm));
 }
 
 __global__ void boys_kernel(int n, const double* __restrict__ T, double* __restrict__ out, const double* __restrict__ tab,
@@ -342,7 +391,7 @@ static mako_status class_flops(mako_pairs p, double thresh, int shard, int nshar
   if ((st = check_pairs(p))) return st;
   if (!(thresh >= 0) || nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "bad args");
   thresh = std::max(thresh, p->tau);
-  if ((st = ensure_plan(p, thresh))) return st;
+  if ((st = ensure_plan(p, thresh, 0.0, nshards))) return st;
   const int NC = NBUCKET * (NBUCKET + 1) / 2;
   fl.assign(NC, 0.0);
   nq.assign(NC, 0);
@@ -356,24 +405,26 @@ static mako_status class_flops(mako_pairs p, double thresh, int shard, int nshar
     const int la = bucket_la(c.X), lb = bucket_lb(c.X), lc = bucket_la(c.Y), ld = bucket_lb(c.Y);
     const double nab = nsph(la) * nsph(lb), ncd = nsph(lc) * nsph(ld);
     const double hab = nH(la + lb), hcd = nH(lc + ld);
-    const long long t0 = shard_cut(c, shard, nshards), t1 = shard_cut(c, shard + 1, nshards);
-    // surviving kets of each (bra, K-group) entry restricted to this shard's tasks
-    for (size_t u = 0; u < c.kbeg.size(); ++u) {
-      const long long a0 = c.task_off[u], a1 = c.task_off[u + 1];
-      if (a1 <= t0 || a0 >= t1) continue;
-      const int Pb = c.ent_P[u];
-      const long long KAB = bx.poff[Pb + 1] - bx.poff[Pb];
-      const int r0 = c.kbeg[u] + (int)(std::max(a0, t0) - a0) * KT;
-      const int r1 = std::min(c.kbeg[u] + (int)(std::min(a1, t1) - a0) * KT, c.kend[u]);
-      if (r1 <= r0) continue;
-      const long long sumK = by.poff[r1] - by.poff[r0];
-      if (!c.swap)
-        fl[ci] += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)sumK * 2.0 * nab * hcd * ncd;
-      else  // task pair = canonical ket (K_CD = KAB here), lanes = canonical bras (sum K_AB = sumK)
-        fl[ci] += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)KAB * (r1 - r0) * 2.0 * nab * hcd * ncd;
-      nq[ci] += r1 - r0;
-      npq[ci] += KAB * sumK;
-    }
+    // surviving kets of each (bra, K-group) entry restricted to this shard's task ranges
+    for_shard_ranges(c, shard, nshards, [&](long long t0, long long t1) {
+      size_t u = std::upper_bound(c.task_off.begin(), c.task_off.end(), t0) - c.task_off.begin() - 1;
+      for (; u < c.kbeg.size() && c.task_off[u] < t1; ++u) {
+        const long long a0 = c.task_off[u], a1 = c.task_off[u + 1];
+        if (a1 <= t0) continue;
+        const int Pb = c.ent_P[u];
+        const long long KAB = bx.poff[Pb + 1] - bx.poff[Pb];
+        const int r0 = c.kbeg[u] + (int)(std::max(a0, t0) - a0) * KT;
+        const int r1 = std::min(c.kbeg[u] + (int)(std::min(a1, t1) - a0) * KT, c.kend[u]);
+        if (r1 <= r0) continue;
+        const long long sumK = by.poff[r1] - by.poff[r0];
+        if (!c.swap)
+          fl[ci] += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)sumK * 2.0 * nab * hcd * ncd;
+        else  // task pair = canonical ket (K_CD = KAB here), lanes = canonical bras (sum K_AB = sumK)
+          fl[ci] += (double)KAB * sumK * 2.0 * nab * hab * hcd + (double)KAB * (r1 - r0) * 2.0 * nab * hcd * ncd;
+        nq[ci] += r1 - r0;
+        npq[ci] += KAB * sumK;
+      }
+    });
   }
   return MAKO_OK;
 }
@@ -483,12 +534,10 @@ extern "C" mako_status mako_build_jk_launches(mako_pairs p, double thresh, int s
   if ((st = check_pairs(p))) return st;
   if (!n || !(thresh >= 0) || nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "bad args");
   thresh = std::max(thresh, p->tau);
-  if ((st = ensure_plan(p, thresh))) return st;
+  if ((st = ensure_plan(p, thresh, 0.0, nshards))) return st;
   int cnt = 1;  // symmetrize
-  for (auto& c : p->plan.cls) {
-    const long long t0 = shard_cut(c, shard, nshards), t1 = shard_cut(c, shard + 1, nshards);
-    if (t1 > t0) ++cnt;
-  }
+  for (auto& c : p->plan.cls)
+    if (c.ntask > 0 && shard_ntask(c.ntask, shard, nshards, shard_chunk(c.ntask, nshards)) > 0) ++cnt;
   *n = cnt;
   return MAKO_OK;
 }
@@ -504,7 +553,7 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
     if (D == J || D == K || J == K) return fail(MAKO_ERR_INVALID, "D, J, K must not alias");
     if (!(thresh >= 0) || !std::isfinite(thresh)) return fail(MAKO_ERR_INVALID, "thresh must be finite and >= 0");
     if (nshards < 1 || shard < 0 || shard >= nshards) return fail(MAKO_ERR_INVALID, "shard out of range");
-    if (flags & ~(unsigned)MAKO_JK_DENSITY_SCREEN) return fail(MAKO_ERR_INVALID, "unknown flags");
+    if (flags & ~(unsigned)(MAKO_JK_DENSITY_SCREEN | MAKO_JK_ACCUMULATE)) return fail(MAKO_ERR_INVALID, "unknown flags");
     const mako_basis_s* B = p->basis;
     const int n = B->nbf;
     cudaStream_t s = (cudaStream_t)cuda_stream;
@@ -512,6 +561,11 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
     const bool dw = (flags & MAKO_JK_DENSITY_SCREEN) != 0;
     const double dw_thresh = std::max(thresh, p->tau);
     double tier_plan = 0.0;
+    // The task counters, the D block maxima and the internal streams are per-handle state: the caller's
+    // stream first waits for the previous build of this handle (which may have been enqueued on another
+    // stream), so two builds in flight on one handle are serialised instead of racing on the counters.
+    if ((st = ensure_streams(p))) return st;
+    for (void* e : p->ev_join) cudaStreamWaitEvent(s, (cudaEvent_t)e, 0);
     if (dw || tier > 0) {
       // shell-block maxima of |D| and the global max; the task plan is the Schwarz prefix at
       // thresh / max|D| rounded down to a power of ten (a superset of the density-screened quartets,
@@ -533,15 +587,20 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
       if (tier > 0) tier_plan = dmax > 0 ? std::pow(10.0, std::floor(std::log10(tier / dmax))) : 0.0;
     }
     thresh = std::max(thresh, p->tau);
-    if ((st = ensure_plan(p, thresh, tier_plan))) return st;
+    if ((st = ensure_plan(p, thresh, tier_plan, nshards))) return st;
     const bool mixed = p->plan.tier > 0.0;
     if (mixed && (st = ensure_lowp(p->set, cuda_stream))) return st;
-    if ((st = cuda_check(cudaMemsetAsync(J, 0, sizeof(double) * n * n, s), "memset J")) ||
-        (st = cuda_check(cudaMemsetAsync(K, 0, sizeof(double) * n * n, s), "memset K")) ||
+    // accumulate mode: the kernels fill per-handle scratch accumulators, added into J/K at the end
+    const bool acc = (flags & MAKO_JK_ACCUMULATE) != 0;
+    const size_t n2 = (size_t)n * n;
+    if (acc && !p->d_jk_scratch.p && (st = p->d_jk_scratch.alloc(2 * sizeof(double) * n2))) return st;
+    double* Jw = acc ? p->d_jk_scratch.as<double>() : J;
+    double* Kw = acc ? p->d_jk_scratch.as<double>() + n2 : K;
+    if ((st = cuda_check(cudaMemsetAsync(Jw, 0, sizeof(double) * n2, s), "memset J")) ||
+        (st = cuda_check(cudaMemsetAsync(Kw, 0, sizeof(double) * n2, s), "memset K")) ||
         (st = cuda_check(cudaMemsetAsync(p->d_counters.p, 0, sizeof(unsigned long long) * 2 * NCLASS, s), "memset ctr")))
       return st;
     int nl = 0;
-    if ((st = ensure_streams(p))) return st;
     // fork: internal streams wait for the zeroed J/K on the caller's stream
     cudaEventRecord((cudaEvent_t)p->ev_fork, s);
     for (void* is : p->streams) cudaStreamWaitEvent((cudaStream_t)is, (cudaEvent_t)p->ev_fork, 0);
@@ -563,9 +622,12 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
       const bool lo = oc.second >= NCL;
       ClassPlan& c = lo ? p->plan.cls_lo[oc.second - NCL] : p->plan.cls[oc.second];
       JKArgs a{};
-      a.task_begin = shard_cut(c, shard, nshards);
-      a.task_end = shard_cut(c, shard + 1, nshards);
-      if (a.task_end <= a.task_begin) continue;
+      a.ntask = c.ntask;
+      a.shard = shard;
+      a.nshards = nshards;
+      a.chunk = nshards == 1 ? c.ntask : shard_chunk(c.ntask, nshards);
+      a.ntask_local = nshards == 1 ? c.ntask : shard_ntask(c.ntask, shard, nshards, a.chunk);
+      if (a.ntask_local <= 0) continue;
       const size_t si = std::min_element(load.begin(), load.end()) - load.begin();
       load[si] += -oc.first;
       cudaStream_t cs = (cudaStream_t)p->streams[si];
@@ -578,11 +640,15 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
       a.ent_P = c.d_ent_P.as<int>();
       a.usamp = c.d_usamp.as<int>();
       a.nent = (int)c.kbeg.size();
+      a.nunit = (int)c.unit_P.size();
+      a.unit_off = c.d_unit_off.as<long long>();
+      a.unit_P = c.d_unit_P.as<int>();
+      a.shl = B->d_l.as<int>();
       a.KT = c.KT;
       a.counter = p->d_counters.as<unsigned long long>() + class_index(c.X, c.Y) + (lo ? NCL : 0);
       a.D = D;
-      a.J = J;
-      a.K = K;
+      a.J = Jw;
+      a.K = Kw;
       a.nbf = n;
       a.ao = B->d_ao.as<int>();
       a.thresh = thresh;
@@ -609,7 +675,8 @@ static mako_status build_jk_impl(mako_pairs p, const double* D, double thresh, d
       cudaEventRecord((cudaEvent_t)p->ev_join[i], (cudaStream_t)p->streams[i]);
       cudaStreamWaitEvent(s, (cudaEvent_t)p->ev_join[i], 0);
     }
-    symmetrize_kernel<<<592, 256, 0, s>>>(J, K, n);
+    if (acc) symmetrize_add_kernel<<<592, 256, 0, s>>>(Jw, Kw, J, K, n);
+    else symmetrize_kernel<<<592, 256, 0, s>>>(J, K, n);
     return cuda_check(cudaGetLastError(), "symmetrize launch");
   } catch (const std::exception& e) {
     return fail(MAKO_ERR_OOM, e.what());
@@ -631,6 +698,32 @@ extern "C" mako_status mako_build_jk_mixed(mako_pairs p, const double* D, double
                                            void* cuda_stream) {
   if (!(thresh_fp64 > 0) || !std::isfinite(thresh_fp64)) return fail(MAKO_ERR_INVALID, "thresh_fp64 must be > 0");
   return build_jk_impl(p, D, thresh, thresh_fp64, flags, J, K, shard, nshards, cuda_stream);
+}
+
+extern "C" mako_status mako_density_delta(mako_pairs p, const double* D, const double* D_prev, double* dD,
+                                          double* dmax, void* cuda_stream) {
+  try {
+    mako_status st;
+    if ((st = check_pairs(p))) return st;
+    if (!D || !D_prev || !dD || !dmax) return fail(MAKO_ERR_INVALID, "NULL argument");
+    if (dD == D || dD == D_prev) return fail(MAKO_ERR_INVALID, "dD must not alias D or D_prev");
+    const int n = p->basis->nbf;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    if (!p->d_dmax.p && (st = p->d_dmax.alloc(sizeof(double)))) return st;
+    if ((st = ensure_streams(p))) return st;
+    for (void* e : p->ev_join) cudaStreamWaitEvent(s, (cudaEvent_t)e, 0);  // d_dmax is per-handle state
+    if ((st = cuda_check(cudaMemsetAsync(p->d_dmax.p, 0, sizeof(double), s), "memset dmax"))) return st;
+    delta_kernel<<<592, 256, 0, s>>>(D, D_prev, dD, (long long)n * n, p->d_dmax.as<unsigned long long>());
+    double h = 0.0;
+    if ((st = cuda_check(cudaMemcpyAsync(&h, p->d_dmax.p, sizeof(double), cudaMemcpyDeviceToHost, s), "dmax")) ||
+        (st = cuda_check(cudaStreamSynchronize(s), "delta sync")))
+      return st;
+    *dmax = h;
+    if (!std::isfinite(h)) return fail(MAKO_ERR_INVALID, "D or D_prev is not finite");
+    return MAKO_OK;
+  } catch (const std::exception& e) {
+    return fail(MAKO_ERR_OOM, e.what());
+  }
 }
 
 extern "C" mako_status mako_class_family(int* family) {
@@ -708,7 +801,9 @@ static mako_status eri_batch_impl(mako_basis basis, int nq, const int* quartets,
         DevBuf& d2 = *keep[keep.size() - 3];
         DevBuf& d3 = *keep[keep.size() - 2];
         DevBuf& d4 = *keep[keep.size() - 1];
-        if ((st = upload(d1, qb)) || (st = upload(d2, qk)) || (st = upload(d3, qf)) || (st = upload(d4, qo))) return st;
+        if ((st = upload_async(d1, qb, s)) || (st = upload_async(d2, qk, s)) || (st = upload_async(d3, qf, s)) ||
+            (st = upload_async(d4, qo, s)))
+          return st;
         BatchArgs a{};
         a.bra = set.b[X].view();
         a.ket = set.b[Y].view();
@@ -750,6 +845,7 @@ extern "C" mako_status mako_boys(int n, const double* T, int mmax, double* out, 
     boys_table(h);
     mako_status st = upload(tab, h);
     if (st) return st;
+    if ((st = cuda_check(cudaDeviceSynchronize(), "boys table upload"))) return st;
     tab_dev = dev;
   }
   boys_kernel<<<(n + 127) / 128, 128, 0, (cudaStream_t)cuda_stream>>>(n, T, out, tab.as<double>(), mmax);

@@ -98,6 +98,11 @@ MK_HD constexpr int kgroup(int K) {
 #ifndef MAKO_KFSWAP_PICK
 #define MAKO_KFSWAP_PICK 302
 #endif
+// warp-per-quartet classes run transposed ((ab|cd) as (cd|ab): the ket side takes the inner, per
+// primitive-quartet GEMM1; S6), measured per class
+#ifndef MAKO_JKSWAP_PICK
+#define MAKO_JKSWAP_PICK -1
+#endif
 #ifndef MAKO_SLAB_PICK
 #define MAKO_SLAB_PICK 202, 402
 #endif
@@ -110,6 +115,7 @@ MK_HD constexpr int kgroup(int K) {
 constexpr int kKfPick[] = {MAKO_KF_PICK};
 constexpr int kKfSwapPick[] = {MAKO_KFSWAP_PICK};
 constexpr int kSlabPick[] = {MAKO_SLAB_PICK};
+constexpr int kJkSwapPick[] = {MAKO_JKSWAP_PICK};
 constexpr int kJkCap4[] = {MAKO_JK_CAP4};
 constexpr int kKfCap3[] = {MAKO_KF_CAP3};
 template <int N>
@@ -122,6 +128,32 @@ MK_HD constexpr bool in_list(const int (&a)[N], int v) {
 // task -> entry lookup: every TASK_SAMPLE-th task's entry is stored, the rest is a short forward scan
 constexpr int TASK_SAMPLE_SHIFT = 4;
 constexpr int TASK_SAMPLE = 1 << TASK_SAMPLE_SHIFT;
+
+#ifndef MAKO_TASK_GRAB
+#define MAKO_TASK_GRAB 4
+#endif
+constexpr int TASK_GRAB = MAKO_TASK_GRAB;  // tasks taken per counter increment (one entry lookup per grab)
+
+// Interleaved shard split: the task index space [0, T) of a class is cut into chunks of
+// C tasks (C a multiple of TASK_GRAB, about 256 chunks per shard); shard s owns chunks j = s, s + n,
+// s + 2n, ...  A pure function of (T, n): every rank derives the same split.
+MK_HD inline long long shard_chunk(long long T, int n) {
+  long long c = T / ((long long)n * 256);
+  c = (c + TASK_GRAB - 1) / TASK_GRAB * TASK_GRAB;
+  return c < 4 * TASK_GRAB ? 4 * TASK_GRAB : c;
+}
+// number of tasks of shard s
+MK_HD inline long long shard_ntask(long long T, int s, int n, long long C) {
+  const long long nch = (T + C - 1) / C;  // chunks, the last one possibly partial
+  if (s >= nch) return 0;
+  const long long mine = (nch - 1 - s) / n + 1;  // chunks s, s+n, ... < nch
+  const long long last = s + (mine - 1) * n;
+  return (mine - 1) * C + ((last == nch - 1) ? T - last * C : C);
+}
+// global task of local task index l of shard s
+MK_HD inline long long shard_task(long long l, int s, int n, long long C) {
+  return ((l / C) * n + s) * C + l % C;
+}
 
 // primitive-pair screening (reading R7)
 constexpr double PRIM_PAIR_EPS = 1e-18;
@@ -148,13 +180,22 @@ struct PairView {
 struct JKArgs {
   PairView bra, ket;
   int same_bucket;
-  long long task_begin, task_end;   // shard range of this class's task index space
+  // shard of the class's task index space [0, ntask): the tasks are cut into chunks of
+  // `chunk` consecutive tasks, chunk j belongs to shard j mod nshards (interleaved, so every shard
+  // samples the whole Q-sorted cost profile of the class); this launch walks its ntask_local tasks
+  long long ntask, ntask_local, chunk;
+  int shard, nshards;
   const long long* task_off;        // [nent+1] task prefix per non-empty (bra pair, ket K-group) entry
   const int* ent_P;                 // [nent] bra pair of the entry
   const int* kbeg;                  // [nent] first ket of the entry (start of its K-group segment)
   const int* kend;                  // [nent] one past the last surviving ket (Q-sorted prefix of the segment)
   const int* usamp;                 // [ntask / TASK_SAMPLE + 1] entry holding task k * TASK_SAMPLE
   int nent;
+  // bra units (strip digestion, eri_tpq.cuh): unit u = tasks [unit_off[u], unit_off[u+1]) of bra pair unit_P[u]
+  int nunit;
+  const long long* unit_off;        // [nunit + 1]
+  const int* unit_P;                // [nunit]
+  const int* shl;                   // [nshell] angular momentum of every shell
   int KT;                           // kets per task
   unsigned long long* counter;      // dynamic task counter (zeroed before launch)
   const double* D;

@@ -66,12 +66,14 @@ struct ClassPlan {
   std::vector<int> ent_P, kbeg, kend;  // [nent] bra pair, first / one-past-last surviving ket
   std::vector<long long> task_off;     // [nent + 1] task prefix
   std::vector<int> usamp;              // [ntask / TASK_SAMPLE + 1] entry holding task k * TASK_SAMPLE
-  std::vector<double> cost_cum;        // [nent + 1] prefix of the modelled cost per entry (shard balance)
-  DevBuf d_ent_P, d_kbeg, d_kend, d_task_off, d_usamp;
+  std::vector<long long> unit_off;     // [nunit + 1] first task of each bra unit (all entries of one bra pair)
+  std::vector<int> unit_P;             // [nunit] bra pair of the unit
+  DevBuf d_ent_P, d_kbeg, d_kend, d_task_off, d_usamp, d_unit_off, d_unit_P;
 };
 
 struct Plan {
   double thresh = -1.0;
+  int nshards = 1;                 // task lengths are sized for the per-shard quartet count
   double tier = 0.0;               // > thresh: reduced-precision tier boundary (0 = FP64 only)
   int KT = 16;
   std::vector<ClassPlan> cls;      // 55 classes (FP64 tier)
@@ -102,6 +104,8 @@ struct mako_pairs_s {
   mako::DevBuf d_counters;      // [2 * NCLASS] task counters (FP64 tier, TF32 tier)
   mako::DevBuf d_dsh;           // [nshell * nshell] float: max |D| per shell block (density screening)
   mako::DevBuf d_dmax;          // [1] double: max |D| (density screening)
+  mako::DevBuf d_jk_scratch;    // [2 * nbf * nbf] accumulators of MAKO_JK_ACCUMULATE builds
+  int nsm = 0;                  // SM count of the pairs' device (task-length sizing)
   // profiling (mako_profile_enable / read)
   bool prof = false;
   // concurrent class launches: internal streams forked from / joined to the caller's stream

@@ -14,14 +14,27 @@ def shard_of(rank, world):
     return int(rank), int(world)
 
 
+def jk_buffer(n, device, dtype=torch.float64):
+    """One preallocated [2, n, n] buffer; J = buf[0] and K = buf[1] are views, so the combine below
+    reduces both in one collective without a staging copy (C5: 8 GB that would otherwise be
+    re-allocated every build)."""
+    buf = torch.empty((2, n, n), dtype=dtype, device=device)
+    return buf, buf[0], buf[1]
+
+
 def combine_jk(J, K, group=None):
-    """Sum the per-rank partial J and K in one collective (packed into one buffer)."""
+    """Sum the per-rank partial J and K in one collective.  When J and K are the two halves of one
+    jk_buffer the all_reduce runs in place on it; otherwise they are reduced one after the other
+    (no temporary)."""
     if not dist.is_initialized() or dist.get_world_size(group) == 1:
         return J, K
-    buf = torch.stack([J, K])
-    dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
-    J.copy_(buf[0])
-    K.copy_(buf[1])
+    base = J._base
+    if (base is not None and base is K._base and base.dim() == 3 and base.shape[0] == 2 and base.is_contiguous()
+            and J.data_ptr() == base.data_ptr() and K.data_ptr() == base[1].data_ptr()):
+        dist.all_reduce(base, op=dist.ReduceOp.SUM, group=group)
+    else:
+        dist.all_reduce(J, op=dist.ReduceOp.SUM, group=group)
+        dist.all_reduce(K, op=dist.ReduceOp.SUM, group=group)
     return J, K
 
 

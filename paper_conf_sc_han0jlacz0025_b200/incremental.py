@@ -19,12 +19,12 @@ SURVEY S8.f row 1; "relaxed precision thresholds during early iter
 quantized kernels - and gradually tightening them as convergence nears"): quartets whose
 contribution bound Q_ab Q_cd max|D_build| is below thresh_fp64_n = precision_scale * max|Delta D_n|
 run the TF32 tier, so the reduced-precision share shrinks as the SCF converges (R21).  All
-device work runs in libmako's kernels; the Delta D / accumulation steps are torch tensor ops
-(plumbing).
+device work runs in libmako's kernels: Delta D and max|Delta D| come from mako_density_delta, the
+update is accumulated into J/K by mako_build_jk_ex / _mixed with MAKO_JK_ACCUMULATE.
 """
 import torch
 
-from .mako import build_jk
+from .mako import build_jk, density_delta
 
 
 def tau_schedule(dmax, tau_final, tau_loose, tau_scale):
@@ -58,6 +58,7 @@ class IncrementalJK:
         self.precision_scale = None if precision_scale is None else float(precision_scale)
         self.device = device or torch.device("cuda")
         self.D = self.J = self.K = None
+        self.dD = None
         self.since_full = 0
         self.tau_full = None
         self.history = []
@@ -71,25 +72,29 @@ class IncrementalJK:
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record()
         if self.D is None:
-            full, dD, dmax = True, Dt, float(Dt.abs().max())
+            self.dD = torch.empty_like(Dt)
+            zero = torch.zeros_like(Dt)
+            _, dmax = density_delta(self.pairs, Dt, zero, self.dD)  # max|D| through the library
+            del zero
         else:
-            dD = (Dt - self.D).contiguous()
-            dmax = float(dD.abs().max())
+            _, dmax = density_delta(self.pairs, Dt, self.D, self.dD)
         tau = tau_schedule(dmax, self.tau_final, self.tau_loose, self.tau_scale)
         full = (self.D is None or self.since_full >= self.rebuild_every or
                 (tau < self.tau_full and (tau <= self.tau_final or tau < self.tighten * self.tau_full)))
         t64 = precision_schedule(dmax, self.precision_scale)
         if full:
-            J, K = build_jk(self.pairs, Dt, thresh=tau, density_screen=True, thresh_fp64=t64)
-            self.J, self.K = J, K
+            if self.J is None:
+                self.J, self.K = torch.empty_like(Dt), torch.empty_like(Dt)
+            build_jk(self.pairs, Dt, thresh=tau, J=self.J, K=self.K, density_screen=True, thresh_fp64=t64)
             self.since_full = 0
             self.tau_full = tau
-        else:
-            dJ, dK = build_jk(self.pairs, dD, thresh=tau, density_screen=True, thresh_fp64=t64)
-            self.J = self.J + dJ
-            self.K = self.K + dK
+        else:  # J += J[dD], K += K[dD] inside the library
+            build_jk(self.pairs, self.dD, thresh=tau, J=self.J, K=self.K, density_screen=True, thresh_fp64=t64,
+                     accumulate=True)
             self.since_full += 1
-        self.D = Dt
+        if self.D is None:
+            self.D = torch.empty_like(Dt)
+        self.D.copy_(Dt)
         ev1.record()
         torch.cuda.synchronize()
         self.history.append({"full": full, "tau": tau, "dmax": dmax, "thresh_fp64": t64, "ms": ev0.elapsed_time(ev1)})

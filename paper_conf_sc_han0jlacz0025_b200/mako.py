@@ -82,6 +82,7 @@ class Pairs:
         h = ctypes.c_void_p()
         check(self._lib.mako_shellpairs_screen(basis.handle, float(tau), _stream_ptr(stream), ctypes.byref(h)))
         self.handle = h
+        self.device = torch.device("cuda", torch.cuda.current_device())
 
     def stats(self, thresh=None):
         a, b, c = ctypes.c_longlong(), ctypes.c_longlong(), ctypes.c_longlong()
@@ -131,29 +132,54 @@ class Pairs:
 
 
 MAKO_JK_DENSITY_SCREEN = 1
+MAKO_JK_ACCUMULATE = 2
 MAKO_ERI_REDUCED = 1
 
 
+def density_delta(pairs, D, D_prev, dD=None, stream=None):
+    """dD = D - D_prev on the device and max|dD| (mako_density_delta; synchronises `stream`)."""
+    if dD is None:
+        dD = torch.empty_like(D)
+    n = pairs.basis.nbf
+    for name, t in (("D", D), ("D_prev", D_prev), ("dD", dD)):
+        if not isinstance(t, torch.Tensor) or tuple(t.shape) != (n, n):
+            raise ValueError(f"{name} must be a {n}x{n} tensor")
+    m = ctypes.c_double()
+    check(pairs._lib.mako_density_delta(pairs.handle, _dev_ptr(D, "D"), _dev_ptr(D_prev, "D_prev"), _dev_ptr(dD, "dD"),
+                                        ctypes.byref(m), _stream_ptr(stream)))
+    return dD, m.value
+
+
 def build_jk(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1, stream=None, density_screen=False,
-             thresh_fp64=None):
+             thresh_fp64=None, accumulate=False):
     """J_{mn} = sum (mn|ls) D_ls, K_{ml} = sum (mn|ls) D_ns on the GPU (north_star).  Async on `stream`
     (density_screen=True: mako_build_jk_ex with MAKO_JK_DENSITY_SCREEN, which synchronises `stream`).
     thresh_fp64: stage-aware reduced-precision build (mako_build_jk_mixed; synchronises `stream`):
-    quartets whose contribution bound Q_ab Q_cd max|D| is below ~thresh_fp64 run the TF32 tier."""
+    quartets whose contribution bound Q_ab Q_cd max|D| is below ~thresh_fp64 run the TF32 tier.
+    accumulate=True: J += J[D], K += K[D] (MAKO_JK_ACCUMULATE; J and K must be given)."""
+    if accumulate and (J is None or K is None):
+        raise ValueError("accumulate=True needs the J and K to accumulate into")
     n = pairs.basis.nbf
-    if D.shape != (n, n):
-        raise ValueError(f"D must be {n}x{n}")
     if J is None:
         J = torch.empty_like(D)
     if K is None:
         K = torch.empty_like(D)
+    # the C ABI takes raw pointers: check shapes and devices here so that an undersized or foreign
+    # buffer is rejected instead of written past its end
+    dev = getattr(pairs, "device", None)
+    for name, t in (("D", D), ("J", J), ("K", K)):
+        if not isinstance(t, torch.Tensor) or tuple(t.shape) != (n, n):
+            raise ValueError(f"{name} must be a {n}x{n} tensor")
+        if dev is not None and t.device != dev:
+            raise ValueError(f"{name} is on {t.device}, the pairs live on {dev}")
     t = float(pairs.tau if thresh is None else thresh)
+    flags = (MAKO_JK_DENSITY_SCREEN if density_screen else 0) | (MAKO_JK_ACCUMULATE if accumulate else 0)
     if thresh_fp64 is not None:
-        check(pairs._lib.mako_build_jk_mixed(pairs.handle, _dev_ptr(D, "D"), t, float(thresh_fp64),
-                                             MAKO_JK_DENSITY_SCREEN if density_screen else 0, _dev_ptr(J, "J"),
-                                             _dev_ptr(K, "K"), int(shard), int(nshards), _stream_ptr(stream)))
-    elif density_screen:
-        check(pairs._lib.mako_build_jk_ex(pairs.handle, _dev_ptr(D, "D"), t, MAKO_JK_DENSITY_SCREEN, _dev_ptr(J, "J"),
+        check(pairs._lib.mako_build_jk_mixed(pairs.handle, _dev_ptr(D, "D"), t, float(thresh_fp64), flags,
+                                             _dev_ptr(J, "J"), _dev_ptr(K, "K"), int(shard), int(nshards),
+                                             _stream_ptr(stream)))
+    elif flags:
+        check(pairs._lib.mako_build_jk_ex(pairs.handle, _dev_ptr(D, "D"), t, flags, _dev_ptr(J, "J"),
                                           _dev_ptr(K, "K"), int(shard), int(nshards), _stream_ptr(stream)))
     else:
         check(pairs._lib.mako_build_jk(pairs.handle, _dev_ptr(D, "D"), t, _dev_ptr(J, "J"), _dev_ptr(K, "K"),

@@ -24,12 +24,22 @@ def _worker(rank, world, port, ret):
 
     def cpu_build(pairs, D, thresh=None, J=None, K=None, shard=0, nshards=1):
         j, k = oracle.jk(sh, D.numpy(), 0.0, shard, nshards)
-        return torch.from_numpy(j), torch.from_numpy(k)
+        if J is None:
+            return torch.from_numpy(j), torch.from_numpy(k)
+        J.copy_(torch.from_numpy(j))
+        K.copy_(torch.from_numpy(k))
+        return J, K
 
+    # separate J, K tensors (two collectives) and one preallocated [2, n, n] buffer (one in-place collective)
     J, K = mdist.distributed_build_jk(None, D, build=cpu_build)
+    buf, Jv, Kv = mdist.jk_buffer(n, "cpu")
+    ptr = buf.data_ptr()
+    J2, K2 = mdist.distributed_build_jk(None, D, J=Jv, K=Kv, build=cpu_build)
+    assert J2.data_ptr() == ptr and K2.data_ptr() == ptr + n * n * 8
     if rank == 0:
         j0, k0 = oracle.jk(sh, D.numpy(), 0.0)
         ret["err"] = float(max(np.abs(J.numpy() - j0).max(), np.abs(K.numpy() - k0).max()))
+        ret["err_buf"] = float(max(np.abs(buf[0].numpy() - j0).max(), np.abs(buf[1].numpy() - k0).max()))
     dist.destroy_process_group()
 
 
@@ -39,3 +49,4 @@ def test_gloo_world2_broadcast_allreduce():
     port = 29500 + os.getpid() % 1000
     mp.spawn(_worker, args=(2, port, ret), nprocs=2, join=True)
     assert ret["err"] < 1e-13
+    assert ret["err_buf"] < 1e-13

@@ -15,8 +15,9 @@ def test_boys_device_vs_oracle():
     import torch
     from paper_conf_sc_han0jlacz0025_b200 import boys
     T = np.concatenate([[0.0, 1e-14, 1e-8, 1e-3], np.linspace(0.01, 45, 3001), [39.99, 40.0, 40.01, 60, 150, 1e4, 1e7]])
-    F = boys(torch.tensor(T, device="cuda"), 12).cpu().numpy()
-    ref = np.array([oracle.boys(12, t) for t in T])
+    # m <= 16: the g classes ((gg|gg), L = 16) run boys_eval<16> (reading R1)
+    F = boys(torch.tensor(T, device="cuda"), 16).cpu().numpy()
+    ref = np.array([oracle.boys(16, t) for t in T])
     err = np.abs(F - ref)
     assert err.max() <= 5e-15, (err.max(), T[np.unravel_index(err.argmax(), err.shape)[0]])
     assert (err / np.maximum(ref, 1e-300)).max() <= 2e-14

@@ -47,6 +47,39 @@ def test_density_screen_vs_oracle_rule():
     assert np.abs(J1 - J2).max() <= 1e-12 * np.abs(J1).max() and np.abs(K1 - K2).max() <= 1e-12 * np.abs(K1).max()
 
 
+def test_accumulate_and_density_delta():
+    """MAKO_JK_ACCUMULATE + mako_density_delta (the incremental update inside the C ABI): J[D1] +
+    J[D2 - D1] equals J[D2] (J, K linear in D); max|dD| is exact; a NaN in D is rejected."""
+    import torch
+    from paper_conf_sc_han0jlacz0025_b200 import MakoError, build_jk, density_delta
+    m, sh, B, P = _setup("benzene-def2svp", 1e-12)
+    n = sh.nbf()
+    D1 = torch.tensor(mi.synthetic_density(n, m.nelec // 2, seed=8), device="cuda")
+    D2 = torch.tensor(mi.synthetic_density(n, m.nelec // 2, seed=9), device="cuda")
+    J, K = build_jk(P, D1)
+    dD, dmax = density_delta(P, D2, D1)
+    torch.cuda.synchronize()
+    ref = (D2 - D1)
+    assert torch.equal(dD, ref) and dmax == float(ref.abs().max())
+    build_jk(P, dD, J=J, K=K, accumulate=True)
+    J2, K2 = build_jk(P, D2)
+    torch.cuda.synchronize()
+    assert float((J - J2).abs().max()) <= 1e-12 * float(J2.abs().max())
+    assert float((K - K2).abs().max()) <= 1e-12 * float(K2.abs().max())
+    # accumulate with density screening and with the mixed build
+    J3, K3 = build_jk(P, D1, density_screen=True, thresh=1e-13)
+    build_jk(P, dD, J=J3, K=K3, density_screen=True, thresh=1e-13, accumulate=True)
+    torch.cuda.synchronize()
+    assert float((J3 - J2).abs().max()) <= 1e-8 and float((K3 - K2).abs().max()) <= 1e-8
+    # non-finite densities fail loudly (NaN survives the block maxima)
+    Dn = D1.clone()
+    Dn[3, 5] = float("nan")
+    with pytest.raises(MakoError):
+        density_delta(P, Dn, D1)
+    with pytest.raises(MakoError):
+        build_jk(P, Dn, density_screen=True)
+
+
 def _scf(mol, sh, jk_fn):
     S, T, V = oracle.one_electron(sh, mol)
     return oracle.rhf(S, T, V, oracle.nuclear_repulsion(mol), mol.nelec // 2, jk_fn)

@@ -99,25 +99,59 @@ def _jk(P, D, **kw):
     return J.cpu().numpy(), K.cpu().numpy()
 
 
+def _reduced_bound(sh, B, Q, D, tau, t64, cap=4e-3):
+    """Per-element error bound of mako_build_jk_mixed vs the FP64 result (readings R20/R21):
+    a quartet (ab|cd) runs the reduced tier iff its class has a reduced kernel and tau <= Q_ab Q_cd < T,
+    T = 10^floor(log10(thresh_fp64 / max|D|)); each of its ERIs is then off by at most cap * Q_ab Q_cd
+    (the ERI-level bar of test_reduced_eri_batch_error_budget, measured <= 8.6e-4).  Summed over the
+    quartets contributing to each element, with |D| weights:
+        |dJ_mn| <= cap sum_{cd reduced} Q_ab Q_cd sum_{l in c, s in d} |D_ls|            (m in a, n in b)
+        |dK_mk| <= cap sum_{b,d: (ab|cd) reduced} Q_ab Q_cd sum_{n in b, s in d} |D_ns|   (m in a, k in c)
+    over ordered shell tuples (every permutation of a canonical quartet contributes once)."""
+    from paper_conf_sc_han0jlacz0025_b200.mako import class_reduced
+    red = class_reduced()
+    ns = sh.nshell
+    off = B.ao_offsets
+    l = np.asarray(sh.l)
+    buck = lambda la, lb: max(la, lb) * (max(la, lb) + 1) // 2 + min(la, lb)
+    bk = np.array([[buck(l[a], l[b]) for b in range(ns)] for a in range(ns)])
+    X = np.maximum(bk[:, :, None, None], bk[None, None, :, :])
+    Y = np.minimum(bk[:, :, None, None], bk[None, None, :, :])
+    cls = X * (X + 1) // 2 + Y
+    dmax = np.abs(D).max()
+    T = 10.0 ** np.floor(np.log10(t64 / dmax))
+    QQ = Q[:, :, None, None] * Q[None, None, :, :]
+    R = red[cls] & (QQ >= tau) & (QQ < T)
+    S1 = np.array([[np.abs(D[off[a]:off[a + 1], off[b]:off[b + 1]]).sum() for b in range(ns)] for a in range(ns)])
+    W = np.where(R, QQ, 0.0)
+    bj = cap * np.einsum("abcd,cd->ab", W, S1)
+    bk_ = cap * np.einsum("abcd,bd->ac", W, S1)
+    exp = lambda m: np.repeat(np.repeat(m, np.diff(off), axis=0), np.diff(off), axis=1)
+    return exp(bj), exp(bk_), int(R.sum())
+
+
 def test_mixed_jk_tiers_vs_oracle():
     m, sh, B, P = _setup("benzene-def2svp", 1e-12)
     D = mi.synthetic_density(sh.nbf(), m.nelec // 2, seed=7)
-    J0, K0 = oracle.jk(sh, D, 1e-12)
+    Q = oracle.schwarz(sh)
+    J0, K0 = oracle.jk(sh, D, 1e-12, Q=Q)
     # no reduced quartets: the FP64 tier reproduces the oracle at the FP64 bar
     J, K = _jk(P, D, thresh_fp64=1e-30)
     assert np.abs(J - J0).max() <= 1e-8 and np.abs(K - K0).max() <= 1e-8
-    dmax = np.abs(D).max()
     prev = 0.0
     for t64 in (1e-8, 1e-6, 1e-4, 1e30):
         J, K = _jk(P, D, thresh_fp64=t64)
-        dj, dk = np.abs(J - J0).max(), np.abs(K - K0).max()
-        print("thresh_fp64 %.0e: max|dJ| %.3e max|dK| %.3e" % (t64, dj, dk))
+        dj, dk = np.abs(J - J0), np.abs(K - K0)
+        bj, bk, nred = _reduced_bound(sh, B, Q, D, 1e-12, t64)
+        print("thresh_fp64 %.0e: %d reduced ordered quartets, max|dJ| %.3e (max bound %.3e), max|dK| %.3e "
+              "(max bound %.3e), worst dJ/bound %.3f dK/bound %.3f" % (
+                  t64, nred, dj.max(), bj.max(), dk.max(), bk.max(), (dj / (bj + 1e-10)).max(),
+                  (dk / (bk + 1e-10)).max()))
         assert np.array_equal(J, J.T) and np.array_equal(K, K.T)
-        # whole-build bound: every element is an FP64 sum of at most nq reduced contributions, each
-        # <= 2 * 4e-3 * min(Q_ab Q_cd max|D|, tier) -- a loose cap; the printed values are what matter
-        assert dj <= 8e-3 * min(t64, 10 * dmax) * 1e3 + 1e-8 and dk <= 8e-3 * min(t64, 10 * dmax) * 1e3 + 1e-8
-        assert max(dj, dk) >= prev * 0.1  # more reduced work -> not dramatically smaller error
-        prev = max(dj, dk)
+        # per element: the reduced-tier bound plus the FP64 bar for the FP64 quartets
+        assert (dj <= bj + 1e-10).all() and (dk <= bk + 1e-10).all()
+        assert max(dj.max(), dk.max()) >= prev * 0.1  # more reduced work -> not dramatically smaller error
+        prev = max(dj.max(), dk.max())
     # fully reduced (every quartet of a reduced class): relative error at the TF32 level
     assert np.abs(J - J0).max() <= 1e-3 * np.abs(J0).max()
 

@@ -197,6 +197,30 @@ def test_eightfold_symmetry_psd_schwarz(pure):
                     assert np.abs(blk).max() <= Q[a, b] * Q[c, d] * (1 + 1e-12)
 
 
+@pytest.mark.parametrize("pure", [True, False])
+def test_schwarz_is_sqrt_of_max_diagonal(pure):
+    """orc_schwarz pinned EXACTLY to its definition (DESIGN reading R6):
+    Q_ab = sqrt(max_{m in a, n in b} |(mn|mn)|) from the full ERI tensor -- a Q taken over all block
+    (mm|nn) or a sum of the diagonal would fail here (it is only an upper bound in the test above).  The
+    maximum over the whole (ab|ab) block equals the diagonal maximum (Cauchy-Schwarz), so that reading
+    is the same definition."""
+    for sh in (_fixed_basis(), _random_basis(4), _random_basis(9)):
+        eri = oracle.eri_full(sh, pure=pure)
+        Q = oracle.schwarz(sh, pure=pure)
+        off = np.concatenate([[0], np.cumsum([(2 * l + 1) if pure else (l + 1) * (l + 2) // 2 for l in sh.l])])
+        wrong = 0
+        for a in range(sh.nshell):
+            for b in range(sh.nshell):
+                diag = [abs(eri[m, n, m, n]) for m in range(off[a], off[a + 1]) for n in range(off[b], off[b + 1])]
+                ref = np.sqrt(max(diag))
+                assert abs(Q[a, b] - ref) <= 1e-14 * ref, (a, b, Q[a, b], ref)
+                blk = eri[off[a]:off[a + 1], off[b]:off[b + 1], off[a]:off[a + 1], off[b]:off[b + 1]]
+                assert abs(np.sqrt(np.abs(blk).max()) - ref) <= 1e-14 * ref
+                mmnn = [abs(eri[m, m, n, n]) for m in range(off[a], off[a + 1]) for n in range(off[b], off[b + 1])]
+                wrong = max(wrong, abs(np.sqrt(max(mmnn)) - ref) / ref)
+        assert wrong > 1e-3  # the (mm|nn) reading differs: the pin discriminates
+
+
 def test_spherical_orthonormal_and_known_forms():
     for l in range(5):
         C = oracle.sph_coeffs(l)
