@@ -166,7 +166,8 @@ mako_status mako_density_delta(mako_pairs pairs, const double* D, const double* 
                                void* cuda_stream);
 /* family[MAKO_NCLASS] (HOST): the kernel family that runs each class (S6): 0 lane-per-ket
  * register kernel, 1 ket-first DMMA kernel, 2 ket-first transposed, 3 slot-batched DMMA kernel,
- * 4 warp-per-quartet DMMA kernel.  For measurement reports. */
+ * 4 warp-per-quartet DMMA kernel, 5 warp-per-quartet transposed ((ab|cd) evaluated as (cd|ab)).
+ * For measurement reports. */
 mako_status mako_class_family(int* family);
 /* mask[MAKO_NCLASS] (HOST): 1 where the class has a reduced-precision (TF32) kernel. */
 mako_status mako_class_reduced(int* mask);

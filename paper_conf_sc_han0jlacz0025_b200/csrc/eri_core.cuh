@@ -53,8 +53,13 @@ struct Cls {
   // R rows kept per bra primitive (computed once per primitive quartet, reused by every row chunk)
   // (d/f x d/f bra pairs are single-primitive in the def2/cc families: no rows to group)
   static constexpr int KR = (LA >= 2 && LB >= 2) ? 1 : clampi(1200 / NH - 1, 1, 4);
+  // batched R (quartet_block_rb): the R rows of up to RB primitive quartets (ket primitive x all bra
+  // primitives) are computed lane-per-quartet in registers (r_regs) and stored at the odd stride RS
+  static constexpr bool RBATCH = L <= 6 && in_list(kRBatchPick, bucket_of(LA, LB) * 100 + bucket_of(LC, LD));
+  static constexpr int RB = 16, RS = NH | 1;
+  static constexpr int W_RCOOP = (KR + 1) * NH > RB * RS || !RBATCH ? (KR + 1) * NH : RB * RS;
   // KR result rows + 1 ping-pong scratch row; doubles as the digestion partial-sum scratch (Ps)
-  static constexpr int W_R = ((KR + 1) * NH > 2 * (NA + NB) * NCD) ? (KR + 1) * NH : 2 * (NA + NB) * NCD;
+  static constexpr int W_R = (W_RCOOP > 2 * (NA + NB) * NCD) ? W_RCOOP : 2 * (NA + NB) * NCD;
   static constexpr int W_V = NAB * NCD; // (ab|cd) block
   static constexpr int W_J = NAB;       // J_ab partial sums over the kets of a task
   static constexpr int W_D = NA * NB + NC * ND + NA * NC + NA * ND + NB * NC + NB * ND;  // staged D blocks
@@ -313,6 +318,138 @@ __device__ __forceinline__ void dmma884(double& c0, double& c1, double a, double
                : "d"(a), "d"(b));
 }
 
+// GEMM1 k-loop of one R row (Eq. 7a): t1[mc][nt] += E~_ab[row chunk ch][p] [p|q] with the B fragment
+// gathered from the R row through htab (a6)
+template <class C>
+__device__ __forceinline__ void gemm1_row(double (&t1)[C::MC][C::NT1][2], const double* __restrict__ E,
+                                          const double* __restrict__ Rr, const uint16_t* __restrict__ htab, int ch,
+                                          int g, int t) {
+#pragma unroll
+  for (int ks = 0; ks < C::KS1; ++ks) {
+    const int pc = 4 * ks + t;
+    double a[C::MC];
+#pragma unroll
+    for (int mc = 0; mc < C::MC; ++mc) {
+      const int row = 8 * (ch * C::MC + mc) + g;
+      a[mc] = (row < C::NAB && pc < C::NHAB) ? __ldg(E + row * C::NHAB + pc) : 0.0;
+    }
+#pragma unroll
+    for (int nt = 0; nt < C::NT1; ++nt) {
+      const int qc = 8 * nt + g;
+      const double b = (pc < C::NHAB && qc < C::NHCD) ? Rr[htab[pc * C::NHCD + qc]] : 0.0;
+#pragma unroll
+      for (int mc = 0; mc < C::MC; ++mc)
+        if (ch * C::MC + mc < C::MT) dmma884(t1[mc][nt][0], t1[mc][nt][1], a[mc], b);
+    }
+  }
+}
+
+// GEMM2 (Eq. 7b / Eq. 11) chained in registers: k-step (nt, e) takes q = 8 nt + 2 t + e from the
+// GEMM1 accumulator of lane (g, t)
+template <class C>
+__device__ __forceinline__ void gemm2_chain(double (&c2)[C::MC][C::NT2][2], const double (&t1)[C::MC][C::NT1][2],
+                                            const double* __restrict__ Ek, int ch, int g, int t) {
+#pragma unroll
+  for (int nt = 0; nt < C::NT1; ++nt)
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const int qq = 8 * nt + 2 * t + e;
+#pragma unroll
+      for (int n2 = 0; n2 < C::NT2; ++n2) {
+        const int cd = 8 * n2 + g;
+        const double b = (qq < C::NHCD && cd < C::NCD) ? __ldg(Ek + qq * C::NCD + cd) : 0.0;
+#pragma unroll
+        for (int mc = 0; mc < C::MC; ++mc)
+          if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
+      }
+    }
+}
+
+template <int L>
+__device__ __forceinline__ void r_regs(double p, double Px, double Py, double Pz, double q, double Qx, double Qy,
+                                       double Qz, const double* __restrict__ btab, double (&R)[nH(L)]);
+
+// Batched-R variant of quartet_block for contracted quartets (K_AB K_CD > 1, K_AB <= RB): per batch of
+// floor(RB / K_AB) ket primitives, lane c computes the whole R^{(0)} of primitive quartet
+// (bra primitive c % K_AB, ket primitive c / K_AB) in registers (Boys + Eq. 5 unrolled, the striped
+// layout of PAPER.md:L233-L237) and stores it to row c of the warp's R rows (the SL -> BL hand-off);
+// the GEMM1 of a ket primitive then runs over all K_AB rows before its single register-chained GEMM2.
+template <class C>
+__device__ void quartet_block_rb(const PairView& bra, int b0, int KAB, const PairView& ket, int k0, int k1,
+                                 double* __restrict__ Rbuf, double* __restrict__ V, const uint16_t* __restrict__ htab,
+                                 const double* __restrict__ btab, int lane) {
+  constexpr int RB = C::RB, RS = C::RS, L = C::L;
+  constexpr bool ONECHUNK = C::NCHUNK == 1 && 2 * C::MC * (C::NT1 + C::NT2) <= 24;
+  const int g = lane >> 2, t = lane & 3;
+  if constexpr (!ONECHUNK)
+    for (int i = lane; i < C::NAB * C::NCD; i += 32) V[i] = 0.0;
+  double c2[C::MC][C::NT2][2];
+#pragma unroll
+  for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+    for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
+  const int nkb = RB / KAB;
+  for (int kb = k0; kb < k1; kb += nkb) {
+    const int nk = min(nkb, k1 - kb);
+    if (lane < nk * KAB) {
+      const int kl = kb + lane / KAB, ij = b0 + lane % KAB;
+      double p, Px, Py, Pz, q, Qx, Qy, Qz;
+      load_pdat<true>(bra.pdat, ij, p, Px, Py, Pz);
+      load_pdat<true>(ket.pdat, kl, q, Qx, Qy, Qz);
+      double Rr[nH(L)];
+      r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, btab, Rr);
+      double* row = Rbuf + lane * RS;
+#pragma unroll
+      for (int h = 0; h < nH(L); ++h) row[h] = Rr[h];
+    }
+    __syncwarp();
+    for (int k = 0; k < nk; ++k) {
+      const double* __restrict__ Ek = ket.Eket + (size_t)(kb + k) * (C::NHCD * C::NCD);
+      for (int ch = 0; ch < C::NCHUNK; ++ch) {
+        double t1[C::MC][C::NT1][2];
+#pragma unroll
+        for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+          for (int nt = 0; nt < C::NT1; ++nt) t1[mc][nt][0] = t1[mc][nt][1] = 0.0;
+        for (int il = 0; il < KAB; ++il)
+          gemm1_row<C>(t1, bra.Ebra + (size_t)(b0 + il) * (C::NAB * C::NHAB), Rbuf + (k * KAB + il) * RS, htab, ch,
+                       g, t);
+        if constexpr (!ONECHUNK) {
+#pragma unroll
+          for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+            for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
+        }
+        gemm2_chain<C>(c2, t1, Ek, ch, g, t);
+        if constexpr (!ONECHUNK) {
+#pragma unroll
+          for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+            for (int n2 = 0; n2 < C::NT2; ++n2)
+#pragma unroll
+              for (int i = 0; i < 2; ++i) {
+                const int row = 8 * (ch * C::MC + mc) + g, col = 8 * n2 + 2 * t + i;
+                if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] += c2[mc][n2][i];
+              }
+        }
+      }
+    }
+    __syncwarp();  // R rows are overwritten by the next batch
+  }
+  if constexpr (ONECHUNK) {
+#pragma unroll
+    for (int mc = 0; mc < C::MC; ++mc)
+#pragma unroll
+      for (int n2 = 0; n2 < C::NT2; ++n2)
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int row = 8 * mc + g, col = 8 * n2 + 2 * t + i;
+          if (row < C::NAB && col < C::NCD) V[row * C::NCD + col] = c2[mc][n2][i];
+        }
+  }
+  __syncwarp();
+}
+
 // (ab|cd) block for bra pair P of `bra` and ket pair R of `ket` into V[ab][cd] (warp SMEM).
 // m8n8k4 f64 fragments (lane = 4g + t): A[g][t]; B[k=t][n=g]; C[g][2t+i].
 // Per ket primitive: R is computed once for up to KR bra primitives into SMEM rows; every row chunk
@@ -329,6 +466,12 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
   const int g = lane >> 2, t = lane & 3;
   const int b0 = __ldg(bra.poff + P), b1 = __ldg(bra.poff + P + 1);
   const int k0 = __ldg(ket.poff + R), k1 = __ldg(ket.poff + R + 1);
+  if constexpr (C::RBATCH) {
+    if ((b1 - b0) * (k1 - k0) > 1 && b1 - b0 <= C::RB) {
+      quartet_block_rb<C>(bra, b0, b1 - b0, ket, k0, k1, Rbuf, V, htab, btab, lane);
+      return;
+    }
+  }
   if constexpr (!ONECHUNK)
     for (int i = lane; i < C::NAB * C::NCD; i += 32) V[i] = 0.0;
   double c2[C::MC][C::NT2][2];
@@ -448,6 +591,21 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
   __syncwarp();
 }
 
+// Orientation of an R x C block of J/K updates in the non-symmetrised accumulators (J = Jacc + Jacc^T,
+// K = Kacc + Kacc^T at the end of the build, so element (r, c) may go to (r, c) or (c, r)): the
+// orientation with the longer contiguous runs (R > C: transposed).  blk_rc maps the y-th element of the
+// block to (r, c) so that consecutive y are adjacent in memory; blk_dst is its accumulator offset.
+template <int R, int C>
+__device__ __forceinline__ void blk_rc(int y, int& r, int& c) {
+  if constexpr (R > C) { c = y / R; r = y % R; }
+  else { r = y / C; c = y % C; }
+}
+template <int R, int C>
+__device__ __forceinline__ size_t blk_dst(int row, int col, int nbf) {
+  if constexpr (R > C) return (size_t)col * nbf + row;
+  else return (size_t)row * nbf + col;
+}
+
 // Digestion of one canonical quartet (north_star J/K; FP64 accumulation).
 // With v' = deg * (ab|cd), deg = 1/2 per coincidence (a=b, c=d, ab=cd), the 8 permutations of a
 // canonical quartet reduce for symmetric D to the 6 forward updates below; the transposed halves
@@ -559,23 +717,32 @@ __device__ void digest(const double* __restrict__ V, double deg, int oa, int ob,
   __syncwarp();
   // 4. K_ac[a][c] = sum_d P_ac[a][c,d] | K_ad[a][d] = sum_c P_ad[a][c,d] |
   //    K_bc[b][c] = sum_d P_bc[b][c,d] | K_bd[b][d] = sum_c P_bd[b][c,d]
+  //    Each block goes to the accumulator in the orientation whose rows are longer (K = Kacc + Kacc^T
+  //    at the end, so either triangle is exact) and consecutive lanes take consecutive columns: one RED
+  //    instruction then covers runs of up to 7 adjacent doubles, and the L2 atomic units work per
+  //    32-byte sector (measured 1.65e11 sectors/s, 4.2e11 doubles/s with 4 doubles per sector,
+  //    tools/atomics_bench.cu)
   constexpr int N1 = NA * NC, N2 = N1 + NA * ND, N3 = N2 + NB * NC, N4 = N3 + NB * ND;
   constexpr int NMX = NC > ND ? NC : ND;
   for (int x = lane; x < N4; x += 32) {
     int base, stride, cnt;
     size_t dst;
     if (x < N1) {
-      const int i = x / NC, k = x % NC;
-      base = DL::PAC + i * NCD + k * ND; stride = 1; cnt = ND; dst = (size_t)(oa + i) * nbf + oc + k;
+      int i, k;
+      blk_rc<NA, NC>(x, i, k);
+      base = DL::PAC + i * NCD + k * ND; stride = 1; cnt = ND; dst = blk_dst<NA, NC>(oa + i, oc + k, nbf);
     } else if (x < N2) {
-      const int i = (x - N1) / ND, l = (x - N1) % ND;
-      base = DL::PAD + i * NCD + l; stride = ND; cnt = NC; dst = (size_t)(oa + i) * nbf + od + l;
+      int i, l;
+      blk_rc<NA, ND>(x - N1, i, l);
+      base = DL::PAD + i * NCD + l; stride = ND; cnt = NC; dst = blk_dst<NA, ND>(oa + i, od + l, nbf);
     } else if (x < N3) {
-      const int j = (x - N2) / NC, k = (x - N2) % NC;
-      base = DL::PBC + j * NCD + k * ND; stride = 1; cnt = ND; dst = (size_t)(ob + j) * nbf + oc + k;
+      int j, k;
+      blk_rc<NB, NC>(x - N2, j, k);
+      base = DL::PBC + j * NCD + k * ND; stride = 1; cnt = ND; dst = blk_dst<NB, NC>(ob + j, oc + k, nbf);
     } else {
-      const int j = (x - N3) / ND, l = (x - N3) % ND;
-      base = DL::PBD + j * NCD + l; stride = ND; cnt = NC; dst = (size_t)(ob + j) * nbf + od + l;
+      int j, l;
+      blk_rc<NB, ND>(x - N3, j, l);
+      base = DL::PBD + j * NCD + l; stride = ND; cnt = NC; dst = blk_dst<NB, ND>(ob + j, od + l, nbf);
     }
     double s = 0.0;
 #pragma unroll

@@ -132,7 +132,11 @@ __device__ __forceinline__ void jk_body(const JKArgs& a) {
       __syncwarp();
     }
     for (int ab = lane; ab < C::NAB; ab += 32)
-      atomicAdd(a.J + (size_t)(oa + ab / C::NB) * a.nbf + ob + ab % C::NB, jab[ab]);
+      {  // J_ab block, oriented for contiguous runs (blk_rc, eri_core.cuh)
+        int i, j;
+        blk_rc<C::NA, C::NB>(ab, i, j);
+        atomicAdd(a.J + blk_dst<C::NA, C::NB>(oa + i, ob + j, a.nbf), jab[i * C::NB + j]);
+      }
     __syncwarp();
   }
   }
@@ -213,7 +217,11 @@ __global__ void __launch_bounds__(CTA_THREADS) jk_kernel_q(JKArgs a) {
       __syncwarp();
     }
     for (int ab = lane; ab < C::NAB; ab += 32)
-      atomicAdd(a.J + (size_t)(oa + ab / C::NB) * a.nbf + ob + ab % C::NB, jab[ab]);
+      {  // J_ab block, oriented for contiguous runs (blk_rc, eri_core.cuh)
+        int i, j;
+        blk_rc<C::NA, C::NB>(ab, i, j);
+        atomicAdd(a.J + blk_dst<C::NA, C::NB>(oa + i, ob + j, a.nbf), jab[i * C::NB + j]);
+      }
     __syncwarp();
   }
   }
@@ -370,10 +378,12 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
       kf_jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, KfCfg<X, Y>::SMEM, cs>>>(a);
     }
   } else if constexpr (use_tpq(X, Y)) {
-    // strip digestion when the bra unit's K rows fit in shared memory (eri_tpq.cuh)
-    static const bool no_strip = std::getenv("MAKO_NO_STRIP") != nullptr;  // A/B experiments only
+    // strip digestion (eri_tpq.cuh) is an experiment, off by default: it cuts the global FP64 atomics
+    // of these classes 5.5x but moves the bound to the shared-memory CAS loops and costs occupancy
+    // (measured 12.32 -> 13.12 s per build, S6); MAKO_STRIP=1 enables it where the strip fits
+    static const bool strip = std::getenv("MAKO_STRIP") != nullptr;
     const size_t ss = tpq_strip_smem<X, Y>(a.nbf, a.nshell);
-    if (!no_strip && a.unit_off && ss <= SMEM_CTA_MAX) {
+    if (strip && a.unit_off && ss <= SMEM_CTA_MAX) {
       const void* fn = a.dsh ? (const void*)tpq_strip_kernel<X, Y, true> : (const void*)tpq_strip_kernel<X, Y>;
       if (set_smem_attr<X, Y>(fn, ss)) return MAKO_ERR_CUDA;
       int nb = 0;

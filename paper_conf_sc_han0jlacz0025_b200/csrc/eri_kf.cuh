@@ -17,6 +17,9 @@
 
 namespace mako {
 
+#ifndef MAKO_KF_EKREG
+#define MAKO_KF_EKREG 0
+#endif
 template <int X, int Y>
 struct KfCfg {
   using C = ClsXY<X, Y>;
@@ -148,6 +151,11 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
         double Rr[nH(L)];
         r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
         const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
+        // small ket E~ (ss, ps kets): the whole matrix with 256-bit loads up front (fewer L1 requests;
+        // the kernel is L1-bound, profiles/README.md); larger ones row by row
+        constexpr bool EK_REG = MAKO_KF_EKREG && NHCD * NCD <= 16;
+        double Ekr[EK_REG ? NHCD : 1][EK_REG ? NCD : 1];
+        if constexpr (EK_REG) load_mat<NHCD, NCD>(ek, Ekr);
         static_for<0, LPK>([&](auto hc) {
           constexpr int H = decltype(hc)::value;
           constexpr int p0 = H * PP, p1 = (p0 + PP < NHAB) ? p0 + PP : NHAB;
@@ -156,7 +164,10 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
               constexpr int qq = decltype(qc)::value;
               double e[NCD];
 #pragma unroll
-              for (int j = 0; j < NCD; ++j) e[j] = __ldg(ek + qq * NCD + j);
+              for (int j = 0; j < NCD; ++j) {
+                if constexpr (EK_REG) e[j] = Ekr[qq][j];
+                else e[j] = __ldg(ek + qq * NCD + j);
+              }
               static_for<p0, p1>([&](auto pc) {
                 constexpr int pp = decltype(pc)::value;
                 constexpr int hs = h_sum(pp, qq);
@@ -242,26 +253,31 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
       constexpr int N1 = NA * NC, N2 = N1 + NA * ND, N3 = N2 + NB * NC, N4 = N3 + NB * ND;
       for (int x = hh; x < N4; x += LPK) {
         double s = 0.0;
+        // (each block in the orientation with contiguous runs over consecutive lanes: blk_rc, eri_core.cuh)
         if (x < N1) {
-          const int i = x / NC, k = x % NC;
+          int i, k;
+          blk_rc<NA, NC>(x, i, k);
           for (int j = 0; j < NB; ++j)
             for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OBD + j * ND + l], s);
-          atomicAdd(a.K + (oa + i) * nb + oc + k, deg * s);
+          atomicAdd(a.K + blk_dst<NA, NC>(oa + i, oc + k, a.nbf), deg * s);
         } else if (x < N2) {
-          const int y = x - N1, i = y / ND, l = y % ND;
+          int i, l;
+          blk_rc<NA, ND>(x - N1, i, l);
           for (int j = 0; j < NB; ++j)
             for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OBC + j * NC + k], s);
-          atomicAdd(a.K + (oa + i) * nb + od + l, deg * s);
+          atomicAdd(a.K + blk_dst<NA, ND>(oa + i, od + l, a.nbf), deg * s);
         } else if (x < N3) {
-          const int y = x - N2, j = y / NC, k = y % NC;
+          int j, k;
+          blk_rc<NB, NC>(x - N2, j, k);
           for (int i = 0; i < NA; ++i)
             for (int l = 0; l < ND; ++l) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OAD + i * ND + l], s);
-          atomicAdd(a.K + (ob + j) * nb + oc + k, deg * s);
+          atomicAdd(a.K + blk_dst<NB, NC>(ob + j, oc + k, a.nbf), deg * s);
         } else {
-          const int y = x - N3, j = y / ND, l = y % ND;
+          int j, l;
+          blk_rc<NB, ND>(x - N3, j, l);
           for (int i = 0; i < NA; ++i)
             for (int k = 0; k < NC; ++k) s = fma(Vk[(i * NB + j) * WS + k * ND + l], Dk[K::OAC + i * NC + k], s);
-          atomicAdd(a.K + (ob + j) * nb + od + l, deg * s);
+          atomicAdd(a.K + blk_dst<NB, ND>(ob + j, od + l, a.nbf), deg * s);
         }
       }
     }

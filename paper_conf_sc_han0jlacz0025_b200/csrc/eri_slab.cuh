@@ -257,7 +257,11 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
       }
     }
     for (int ab = lane; ab < NAB; ab += 32)
-      atomicAdd(a.J + (size_t)(oa + ab / C::NB) * a.nbf + ob + ab % C::NB, jab[ab]);
+      {  // J_ab block, oriented for contiguous runs (blk_rc, eri_core.cuh)
+        int i, j;
+        blk_rc<C::NA, C::NB>(ab, i, j);
+        atomicAdd(a.J + blk_dst<C::NA, C::NB>(oa + i, ob + j, a.nbf), jab[i * C::NB + j]);
+      }
     __syncwarp();
   }
   }

@@ -169,11 +169,49 @@ struct Strip {
 // shared-memory double add (sm_100a has no native f64 shared atomic: CAS loop, rarely contended here)
 __device__ __forceinline__ void sh_add(double* p, double v) { atomicAdd(p, v); }
 
+// Sector-grouped digestion of one R x C block per lane (lane = ket) of the lane-per-ket kernel: the
+// lanes' block values go through warp shared memory so that each RED instruction covers, for ~32/run
+// kets, a run of adjacent doubles (the block orientation with the longer runs, blk_rc / blk_dst in
+// eri_core.cuh): the L2 atomic units are bound per 32-byte sector, not per double (1.65e11 sectors/s
+// measured, tools/atomics_bench.cu), and the direct per-lane atomics hit one sector per double.
+#ifndef MAKO_TPQ_STAGE
+#define MAKO_TPQ_STAGE 1
+#endif
+template <int R, int CC, class F>
+__device__ __forceinline__ void staged_red(double* __restrict__ out, double* __restrict__ stage, int lane, bool active,
+                                           int orow, int ocol, int nbf, F&& val) {
+  constexpr int E = R * CC;
+#pragma unroll
+  for (int y = 0; y < E; ++y) {
+    int r, c;
+    blk_rc<R, CC>(y, r, c);
+    stage[lane * E + y] = active ? val(r, c) : 0.0;
+  }
+  __syncwarp();
+#pragma unroll
+  for (int it = 0; it < E; ++it) {
+    const int idx = it * 32 + lane, ket = idx / E, y = idx % E;
+    const int orw = __shfl_sync(0xffffffffu, orow, ket), ocl = __shfl_sync(0xffffffffu, ocol, ket);
+    const double v = stage[idx];
+    int r, c;
+    blk_rc<R, CC>(y, r, c);
+    if (v != 0.0) atomicAdd(out + blk_dst<R, CC>(orw + r, ocl + c, nbf), v);
+  }
+  __syncwarp();
+}
+template <class C>
+__host__ __device__ constexpr int tpq_stage_doubles() {
+  constexpr int a = C::NA * C::NC, b = C::NA * C::ND, c = C::NB * C::NC, d = C::NB * C::ND, e = C::NC * C::ND;
+  constexpr int m1 = a > b ? a : b, m2 = c > d ? c : d, m3 = m1 > m2 ? m1 : m2;
+  return 32 * (m3 > e ? m3 : e);
+}
+
 // One lane-per-ket task: bra pair P, kets [r0, r1) (<= 32, lane i takes ket r0 + i).  Boys, R, the
 // ket-first contraction and digestion all in registers.  STRIP: the K_ac/K_ad/K_bc/K_bd updates and
 // J_ab go to the CTA's shared K-row strip of bra P instead of global FP64 atomics (J_cd stays global).
 template <int X, int Y, bool DW, bool STRIP>
-__device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1, int lane, const Strip& st) {
+__device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1, int lane, const Strip& st,
+                                         double* __restrict__ stage = nullptr) {
   using C = ClsXY<X, Y>;
   constexpr int NAB = C::NAB, NCD = C::NCD, NHAB = C::NHAB, NHCD = C::NHCD, L = C::L;
   constexpr int NA = C::NA, NB = C::NB, NC = C::NC, ND = C::ND;
@@ -297,6 +335,49 @@ __device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1,
         else atomicAdd(a.J + (oa + i / NB) * n + ob + i % NB, 2.0 * s);
       }
     }
+    if constexpr (!STRIP && MAKO_TPQ_STAGE) {
+      const double* __restrict__ Db = Dm;
+      // J_cd ; K_ac += v D_bd ; K_ad += v D_bc ; K_bc += v D_ad ; K_bd += v D_ac (deg = 0 on idle lanes)
+      staged_red<NC, ND>(a.J, stage, lane, active, oc, od, a.nbf, [&](int k, int l) {
+        double s = 0.0;
+#pragma unroll
+        for (int ij = 0; ij < NAB; ++ij) s = fma(V[ij][k * ND + l], __ldg(Db + (oa + ij / NB) * n + ob + ij % NB), s);
+        return 2.0 * deg * s;
+      });
+      staged_red<NA, NC>(a.K, stage, lane, active, oa, oc, a.nbf, [&](int i, int k) {
+        double s = 0.0;
+#pragma unroll
+        for (int j = 0; j < NB; ++j)
+#pragma unroll
+          for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Db + (ob + j) * n + od + l), s);
+        return deg * s;
+      });
+      staged_red<NA, ND>(a.K, stage, lane, active, oa, od, a.nbf, [&](int i, int l) {
+        double s = 0.0;
+#pragma unroll
+        for (int j = 0; j < NB; ++j)
+#pragma unroll
+          for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Db + (ob + j) * n + oc + k), s);
+        return deg * s;
+      });
+      staged_red<NB, NC>(a.K, stage, lane, active, ob, oc, a.nbf, [&](int j, int k) {
+        double s = 0.0;
+#pragma unroll
+        for (int i = 0; i < NA; ++i)
+#pragma unroll
+          for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Db + (oa + i) * n + od + l), s);
+        return deg * s;
+      });
+      staged_red<NB, ND>(a.K, stage, lane, active, ob, od, a.nbf, [&](int j, int l) {
+        double s = 0.0;
+#pragma unroll
+        for (int i = 0; i < NA; ++i)
+#pragma unroll
+          for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Db + (oa + i) * n + oc + k), s);
+        return deg * s;
+      });
+      return;
+    }
     if (!active) return;
     // J_cd
 #pragma unroll
@@ -373,6 +454,8 @@ __device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1,
 template <int X, int Y, bool DW = false>
 __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
   const int lane = threadIdx.x & 31;
+  __shared__ double stage_all[MAKO_TPQ_STAGE ? 4 * tpq_stage_doubles<ClsXY<X, Y>>() : 1];
+  double* stage = stage_all + (MAKO_TPQ_STAGE ? (threadIdx.x >> 5) * tpq_stage_doubles<ClsXY<X, Y>>() : 0);
   for (;;) {
   long long tg0, tg1;
   if (!grab_tasks(a, lane, tg0, tg1)) break;
@@ -382,7 +465,7 @@ __global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
     const int P = __ldg(a.ent_P + U);
     const int r0 = __ldg(a.kbeg + U) + (int)(task - __ldg(a.task_off + U)) * 32;
     const int r1 = min(r0 + 32, __ldg(a.kend + U));
-    tpq_task<X, Y, DW, false>(a, P, r0, r1, lane, Strip{});
+    tpq_task<X, Y, DW, false>(a, P, r0, r1, lane, Strip{}, stage);
   }
   }
 }

@@ -101,10 +101,10 @@ MK_HD constexpr int kgroup(int K) {
 // warp-per-quartet classes run transposed ((ab|cd) as (cd|ab): the ket side takes the inner, per
 // primitive-quartet GEMM1; S6), measured per class
 #ifndef MAKO_JKSWAP_PICK
-#define MAKO_JKSWAP_PICK -1
+#define MAKO_JKSWAP_PICK 703, 803, 706, 503, 802, 806, 901, 804, 502, 807, 504, 906, 903, 907, 702, 904, 805, 902
 #endif
 #ifndef MAKO_SLAB_PICK
-#define MAKO_SLAB_PICK 202, 402
+#define MAKO_SLAB_PICK 402
 #endif
 #ifndef MAKO_JK_CAP4
 #define MAKO_JK_CAP4 800, 801, 802, 803, 804, 805, 806, 807, 808, 705
@@ -116,6 +116,12 @@ constexpr int kKfPick[] = {MAKO_KF_PICK};
 constexpr int kKfSwapPick[] = {MAKO_KFSWAP_PICK};
 constexpr int kSlabPick[] = {MAKO_SLAB_PICK};
 constexpr int kJkSwapPick[] = {MAKO_JKSWAP_PICK};
+// warp-per-quartet classes (codes bucket(la,lb) * 100 + bucket(lc,ld) of the evaluated orientation)
+// whose contracted quartets take the batched lane-per-quartet R path (eri_core.cuh quartet_block_rb)
+#ifndef MAKO_RBATCH_PICK
+#define MAKO_RBATCH_PICK 207, 205, 602, 404, 202
+#endif
+constexpr int kRBatchPick[] = {MAKO_RBATCH_PICK};
 constexpr int kJkCap4[] = {MAKO_JK_CAP4};
 constexpr int kKfCap3[] = {MAKO_KF_CAP3};
 template <int N>

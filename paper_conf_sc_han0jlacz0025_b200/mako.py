@@ -195,7 +195,7 @@ def class_reduced():
 
 
 FAMILY_KERNELS = {0: "tpq_jk_kernel", 1: "kf_jk_kernel", 2: "kf_jk_kernel (transposed)", 3: "slab_jk_kernel",
-                  4: "jk_kernel"}
+                  4: "jk_kernel", 5: "jk_kernel (transposed)"}
 
 
 def class_family():

@@ -71,7 +71,7 @@ def test_production_kernels_eri_columns_spdf(seed):
     """Every l <= 3 class through the production kernel of its family; K in {1, 3} primitives."""
     from paper_conf_sc_han0jlacz0025_b200.mako import class_family
     fam = class_family()
-    assert set(fam[:55]) == {0, 1, 2, 3, 4}  # all five families appear among the l <= 3 classes
+    assert {0, 1, 2, 3, 4, 5} <= set(fam[:55])  # every family appears among the l <= 3 classes
     sh, Z, xyz = _basis(3, 3, (1, 3), seed)
     wj, wk = _columns(sh, Z, xyz)
     print("spdf production kernels: max |dERI| via J %.2e, via K %.2e" % (wj, wk))

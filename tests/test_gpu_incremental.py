@@ -111,40 +111,100 @@ def test_incremental_scf_energies():
 
 
 @pytest.mark.skipif(not os.environ.get("MAKO_SCF_TIMING"), reason="timing run (MAKO_SCF_TIMING=1)")
-def test_incremental_scf_timing():
-    """(Gly)10 def2-SVP RHF: per-iteration device time of plain vs incremental density-screened
-    J/K builds (the measurement of SURVEY S8.f row 2); written to gpurun_out/scf_timing.json."""
+@pytest.mark.parametrize("cfg", ["benzene-def2svp", "gly10-def2svp"])
+def test_scf_timing_line(cfg):
+    """Measurement line of a full RHF on the GPU J/K (BASELINE configs[1] benzene def2-SVP "full SCF";
+    gly10-def2svp = the polyglycine family of PAPER.md Fig. 8 for the row-f2 comparison), written to
+    gpurun_out/scf_<cfg>.json in bench.py's JSON format.  Two SCF runs with the same driver:
+      plain        mako_build_jk on D_n every iteration (the value / s_per_iter of the line);
+      incremental  IncrementalJK: Delta D builds with density-weighted screening, accumulated in the
+                   library, convergence-aware threshold (row f2).
+    s/iter = mean device time of the J/K build per SCF iteration excluding the first.
+    The oracle RHF (same driver, oracle J/K) gives dE and the cpu_baseline (benzene only: the oracle
+    J/K of (Gly)10 takes minutes per iteration).  H, S and the SCF driver are test support (oracle/)."""
     import time
     import torch
+    import bench
     from paper_conf_sc_han0jlacz0025_b200 import IncrementalJK, build_jk
-    m, sh, B, P = _setup(os.environ.get("MAKO_SCF_CONFIG", "gly10-def2svp"), 1e-12)
+    from paper_conf_sc_han0jlacz0025_b200.mako import FAMILY_KERNELS, class_family
+    m, sh, B, P = _setup(cfg, 1e-12)
+    n = sh.nbf()
     S, T, V = oracle.one_electron(sh, m)
     enuc = oracle.nuclear_repulsion(m)
-    plain_ms = []
+    nocc = m.nelec // 2
+    flops = P.flops()["gemm_flops"]
+    cls_flops, _ = P.class_flops()
+    Dd = torch.empty((n, n), dtype=torch.float64, device="cuda")
+    J, K = torch.empty_like(Dd), torch.empty_like(Dd)
+    ms = []
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 
     def plain(D):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        Dt = torch.tensor(D, device="cuda")
-        e0.record()
-        J, K = build_jk(P, Dt)
-        e1.record()
+        Dd.copy_(torch.from_numpy(D))
+        ev0.record()
+        build_jk(P, Dd, J=J, K=K)
+        ev1.record()
         torch.cuda.synchronize()
-        plain_ms.append(e0.elapsed_time(e1))
+        ms.append(ev0.elapsed_time(ev1))
         return J.cpu().numpy(), K.cpu().numpy()
 
-    t0 = time.time()
-    r_plain = oracle.rhf(S, T, V, enuc, m.nelec // 2, plain, e_tol=1e-9, d_tol=1e-6)
-    t1 = time.time()
+    plain(np.zeros((n, n)))  # warm-up (plan, first launches)
+    ms.clear()
+    clocks = bench.ClockSampler(0)
+    clocks.start()
+    P.profile(True)
+    t0 = time.perf_counter()
+    r_plain = oracle.rhf(S, T, V, enuc, nocc, plain, e_tol=1e-10, d_tol=1e-8)
+    t1 = time.perf_counter()
+    cls_ms, cls_n = P.profile_read()
+    P.profile(False)
     inc = IncrementalJK(P)
-    r_inc = oracle.rhf(S, T, V, enuc, m.nelec // 2, inc, e_tol=1e-9, d_tol=1e-6)
-    t2 = time.time()
-    out = {"config": os.environ.get("MAKO_SCF_CONFIG", "gly10-def2svp"), "nbf": sh.nbf(),
-           "plain": {"energy": r_plain.energy, "iterations": r_plain.iterations, "build_ms": plain_ms,
-                     "wall_s": t1 - t0},
-           "incremental": {"energy": r_inc.energy, "iterations": r_inc.iterations, "builds": inc.history,
-                           "wall_s": t2 - t1},
-           "dE": r_inc.energy - r_plain.energy}
+    r_inc = oracle.rhf(S, T, V, enuc, nocc, inc, e_tol=1e-10, d_tol=1e-8)
+    t2 = time.perf_counter()
+    clk = clocks.stop()
+    inc_ms = [h["ms"] for h in inc.history]
+    plain_s = float(np.mean(ms[1:])) * 1e-3
+    inc_s = float(np.mean(inc_ms[1:])) * 1e-3
+    pk = bench.peaks()
+    c = int(np.argmax(cls_ms))
+    ach = cls_flops[c] / (cls_ms[c] / max(cls_n[c], 1) * 1e-3) / 1e12
+    X = int((np.sqrt(8 * c + 1) - 1) // 2)
+    Y = c - X * (X + 1) // 2
+    nm = ["ss", "ps", "pp", "ds", "dp", "dd", "fs", "fp", "fd", "ff", "gs", "gp", "gd", "gf", "gg"]
+    out = {"metric": bench.METRIC, "value": flops / plain_s / 1e12, "unit": bench.UNIT, "n_gpus": 1,
+           "steps": len(ms), "warmup": 1, "ms_per_step": plain_s * 1e3, "higher_is_better": True,
+           "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+           "config": {"workload": cfg + "-rhf", "basis": mi.basis_label(mi.config_molecule(cfg)[1]), "nbf": n,
+                      "shells": sh.nshell, "tau": 1e-12, "gemm_flops_per_build": flops},
+           "s_per_iter": plain_s, "clocks": clk,
+           "roofline": {"bound": "tensor", "achieved": ach, "peak": pk["dmma_m16n8k4_tflops"], "unit": "TFLOP/s",
+                        "frac": ach / pk["dmma_m16n8k4_tflops"], "traffic": None,
+                        "kernel": f"{FAMILY_KERNELS[int(class_family()[c])]} class ({nm[X]}|{nm[Y]})",
+                        "share_of_step": float(cls_ms[c] / max(cls_ms.sum(), 1e-9))},
+           "scf": {"plain": {"energy": r_plain.energy, "iterations": r_plain.iterations,
+                             "converged": r_plain.converged, "build_s_per_iter_excl_first": plain_s,
+                             "wall_s_per_iter": (t1 - t0) / r_plain.iterations},
+                   "incremental": {"energy": r_inc.energy, "iterations": r_inc.iterations,
+                                   "converged": r_inc.converged, "build_s_per_iter_excl_first": inc_s,
+                                   "wall_s_per_iter": (t2 - t1) / r_inc.iterations,
+                                   "full_builds": int(sum(h["full"] for h in inc.history)),
+                                   "build_ms": inc_ms, "tau_per_build": [h["tau"] for h in inc.history]},
+                   "speedup_incremental": plain_s / inc_s,
+                   "dE_incremental_vs_plain": r_inc.energy - r_plain.energy,
+                   "support": "H, S, guess, DIIS: oracle/ (test support); J/K: libmako"}}
+    if cfg == "benzene-def2svp":
+        t3 = time.perf_counter()
+        r_orc = oracle.rhf(S, T, V, enuc, nocc, lambda D: oracle.jk(sh, D, 1e-12), e_tol=1e-10, d_tol=1e-8)
+        t4 = time.perf_counter()
+        out["scf"]["oracle"] = {"energy": r_orc.energy, "iterations": r_orc.iterations,
+                                "wall_s_per_iter": (t4 - t3) / r_orc.iterations}
+        out["scf"]["dE_plain_vs_oracle"] = r_plain.energy - r_orc.energy
+        out["cpu_baseline"] = {"value": flops / ((t4 - t3) / r_orc.iterations) / 1e12, "unit": bench.UNIT,
+                               "cores": oracle.num_threads(), "kind": "oracle",
+                               "sample": "the full oracle RHF (oracle J/K every iteration), wall per iteration"}
+        assert abs(r_plain.energy - r_orc.energy) <= 1e-7
     os.makedirs("gpurun_out", exist_ok=True)
-    json.dump(out, open("gpurun_out/scf_timing.json", "w"), indent=1)
-    print(json.dumps({k: v for k, v in out.items() if k != "incremental"})[:500])
+    json.dump(out, open(f"gpurun_out/scf_{cfg}.json", "w"), indent=1)
+    print(json.dumps({k: v for k, v in out.items() if k != "scf"}))
+    assert r_plain.converged and r_inc.converged
     assert abs(r_inc.energy - r_plain.energy) <= 1e-7
