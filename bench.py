@@ -159,39 +159,44 @@ class ClockSampler:
 # ---------------------------------------------------------------------------------------------
 # CPU baseline: the oracle as it stands, on a bounded sample of the same workload
 # ---------------------------------------------------------------------------------------------
-def oracle_overhead(sh, D, tau, Q):
-    """Per-call cost of oracle.jk that does not scale with the sample (per-thread nbf^2 accumulators,
-    their reduction, the symmetrisation): one call on an empty shard (no bra pair has index % S == S-1
-    when S > npair).  A full build pays it once."""
-    import oracle
+def _nquartet_index(sh):
     npair = sh.nshell * (sh.nshell + 1) // 2
+    return npair * (npair + 1) // 2  # canonical quartet indices P(P+1)/2 + R, R <= P < npair
+
+
+def oracle_overhead(sh, D, tau, Q):
+    """Per-call cost of the oracle J/K that does not scale with the sample (per-thread nbf^2 accumulators,
+    their reduction, the symmetrisation): one call on an empty quartet sample (shard index beyond the
+    last canonical quartet).  A full build pays it once."""
+    import oracle
+    nidx = _nquartet_index(sh)
     t0 = time.perf_counter()
-    oracle.jk(sh, D, tau, npair, npair + 1, Q=Q)
+    oracle.jk_qsample(sh, D, tau, nidx, nidx + 1, Q=Q)
     return time.perf_counter() - t0
 
 
 def oracle_sample_seconds(sh, D, tau, Q, target_s, first_shard=0):
-    """Size a strided sample of canonical bra pairs (index % S == shard) so that its WORK (call time
-    minus the per-call overhead) is about target_s; returns (S, overhead_s).  The pilot uses 8 spread
-    shards of 1/S0 so that one atypical pair does not set the size."""
+    """Size a uniform quartet sample (canonical quartet index % S == shard, orc_jk_qsample: every class and
+    every bra pair sampled alike, so the spread between samples is small) so that its WORK (call time
+    minus the per-call overhead) is about target_s; returns (S, overhead_s).  S < 2: the whole build fits."""
     import oracle
-    npair = sh.nshell * (sh.nshell + 1) // 2
+    nidx = _nquartet_index(sh)
     ovh = oracle_overhead(sh, D, tau, Q)
-    S0 = max(2, min(npair, 20000))
+    S0 = max(2, min(nidx, 40000))  # pilot samples of a few seconds: the work dominates the overhead
     t0 = time.perf_counter()
-    for i in range(8):
-        oracle.jk(sh, D, tau, (first_shard + (i * S0) // 8 + 1) % S0, S0, Q=Q)
-    work = max((time.perf_counter() - t0) / 8 - ovh, 1e-4)
-    S = int(min(work * S0 / target_s, npair))  # S < 2: the full build fits the budget
+    for i in range(2):
+        oracle.jk_qsample(sh, D, tau, (first_shard + i * (S0 // 2) + 1) % S0, S0, Q=Q)
+    work = max((time.perf_counter() - t0) / 2 - ovh, 1e-4)
+    S = int(min(work * S0 / target_s, nidx))
     return S, ovh
 
 
 def oracle_sampled_build(sh, D, tau, Q, S, shard, ovh):
-    """One timed oracle call on the sample shard/S; extrapolated full-build seconds
+    """One timed oracle call on the quartet sample shard/S; extrapolated full-build seconds
     (work x S + the per-call overhead once)."""
     import oracle
     t0 = time.perf_counter()
-    oracle.jk(sh, D, tau, shard, S, Q=Q)
+    oracle.jk_qsample(sh, D, tau, shard, S, Q=Q)
     ts = time.perf_counter() - t0
     return ts, max(ts - ovh, 0.0) * S + ovh
 
@@ -210,8 +215,9 @@ def cpu_baseline(sh, D, tau, total_flops, target_s=15.0, Q=None):
     shard = S // 2
     ts, s_per_build = oracle_sampled_build(sh, D, tau, Q, S, shard, ovh)
     return {"value": total_flops / s_per_build / 1e12, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"canonical bra pairs with pair_index % {S} == {shard} (1/{S} of the build): {ts:.1f} s "
-                      f"measured, per-call overhead {ovh:.2f} s (empty-shard call) counted once, work x{S}",
+            "sample": f"canonical shell quartets with quartet_index % {S} == {shard} (1/{S} of the build, every "
+                      f"class sampled uniformly): {ts:.1f} s measured, per-call overhead {ovh:.2f} s (empty-sample "
+                      f"call) counted once, work x{S}",
             "s_per_iter_extrapolated": s_per_build, "sample_s": ts, "overhead_s": ovh, "extrapolated": True}
 
 
@@ -249,9 +255,9 @@ def run_reference(args):
                        "quartets": nq, "gemm_flops_per_build": total},
             "s_per_iter": s_per_build,
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
-                             "sample": f"each step: canonical bra pairs with index % {S} == shard (1/{S} of the "
-                                       f"build, shards vary per step; {np.mean(samples):.1f} s measured per step), "
-                                       f"work x{S} + per-call overhead {ovh:.2f} s once (extrapolated)"},
+                             "sample": f"each step: canonical shell quartets with index % {S} == shard (1/{S} of "
+                                       f"the build, shards vary per step; {np.mean(samples):.1f} s measured per "
+                                       f"step), work x{S} + per-call overhead {ovh:.2f} s once (extrapolated)"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -455,8 +461,9 @@ def main():
     ap.add_argument("--config", default=DEFAULT_CONFIG, choices=sorted(mi.CONFIGS))
     ap.add_argument("--tau", type=float, default=TAU)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=15.0)
-    ap.add_argument("--ref-step-s", type=float, default=6.0)
+    # both CPU legs size their quartet sample with the same target, so their extrapolations agree
+    ap.add_argument("--cpu-seconds", type=float, default=8.0)
+    ap.add_argument("--ref-step-s", type=float, default=8.0)
     ap.add_argument("--class-times", action="store_true")
     ap.add_argument("--mixed", type=float, default=1e-6,
                     help="thresh_fp64 of the reduced-precision measurement (0 = skip)")

@@ -542,12 +542,21 @@ static void digest(const basis_t* B, int a, int b, int c, int d, const double* b
    (an oracle-side sample; the GPU library's own shard partition is not replicated here).
    Qin: optional precomputed Schwarz table (orc_schwarz), NULL to compute it here.
    J, K: [nbf][nbf] outputs (overwritten), final symmetrised values. */
-static int jk_impl(BASIS_ARGS, const double* Dm, double tau, double tau_dw, int shard, int nshards,
-                   const double* Qin, double* Jout, double* Kout);
+static int jk_impl(BASIS_ARGS, const double* Dm, double tau, double tau_dw, long long shard, long long nshards,
+                   int qsample, const double* Qin, double* Jout, double* Kout);
 
 int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, const double* Qin, double* Jout,
            double* Kout) {
-  return jk_impl(nshell, l, nprim, xyz, exps, coefs, pure, Dm, tau, -1.0, shard, nshards, Qin, Jout, Kout);
+  return jk_impl(nshell, l, nprim, xyz, exps, coefs, pure, Dm, tau, -1.0, shard, nshards, 0, Qin, Jout, Kout);
+}
+
+/* Quartet-level sample (for timing the oracle on a bounded part of a large build; bench.py cpu_baseline):
+   as orc_jk, but the canonical quartet (P, R), R <= P (pair index P = a(a+1)/2 + b), is evaluated iff
+   (P(P+1)/2 + R) % nshards == shard.  Every bra pair and every class is sampled uniformly, so the work
+   of one shard is 1/nshards of the build with a small spread; the shards sum to orc_jk (same J/K). */
+int orc_jk_qsample(BASIS_ARGS, const double* Dm, double tau, long long shard, long long nshards, const double* Qin,
+                   double* Jout, double* Kout) {
+  return jk_impl(nshell, l, nprim, xyz, exps, coefs, pure, Dm, tau, -1.0, shard, nshards, 1, Qin, Jout, Kout);
 }
 
 /* Density-weighted screening ("density-weighted Schwarz"; reading R17):
@@ -556,11 +565,11 @@ int orc_jk(BASIS_ARGS, const double* Dm, double tau, int shard, int nshards, con
 int orc_jk_dw(BASIS_ARGS, const double* Dm, double tau, double tau_dw, const double* Qin, double* Jout,
               double* Kout) {
   if (!(tau_dw >= 0)) return 1;
-  return jk_impl(nshell, l, nprim, xyz, exps, coefs, pure, Dm, tau, tau_dw, 0, 1, Qin, Jout, Kout);
+  return jk_impl(nshell, l, nprim, xyz, exps, coefs, pure, Dm, tau, tau_dw, 0, 1, 0, Qin, Jout, Kout);
 }
 
-static int jk_impl(BASIS_ARGS, const double* Dm, double tau, double tau_dw, int shard, int nshards,
-                   const double* Qin, double* Jout, double* Kout) {
+static int jk_impl(BASIS_ARGS, const double* Dm, double tau, double tau_dw, long long shard, long long nshards,
+                   int qsample, const double* Qin, double* Jout, double* Kout) {
   BASIS_INIT(B);
   if (nshards < 1 || shard < 0 || shard >= nshards || tau < 0) { basis_free(&B); return 1; }
   int N = B.nbf;
@@ -598,9 +607,14 @@ static int jk_impl(BASIS_ARGS, const double* Dm, double tau, double tau_dw, int 
     double* blk = (double*)malloc(sizeof(double) * 81 * 81 * 81 * 81 / 81);
 #pragma omp for schedule(dynamic, 1)
     for (int P = 0; P < npair; ++P) {
-      if (P % nshards != shard) continue;
+      if (!qsample && P % nshards != shard) continue;
       int a = pa[P], b = pb[P];
-      for (int R = 0; R <= P; ++R) {
+      /* quartet sample: first R with (P(P+1)/2 + R) % nshards == shard, then every nshards-th */
+      const long long base = (long long)P * (P + 1) / 2;
+      const long long R0 = qsample ? ((shard - base % nshards) % nshards + nshards) % nshards : 0;
+      if (R0 > P) continue;  /* no quartet of this bra pair in the sample */
+      const int Rstep = qsample ? (int)(nshards < (long long)npair + 1 ? nshards : (long long)npair + 1) : 1;
+      for (int R = (int)R0; R <= P; R += Rstep) {
         int c = pa[R], d = pb[R];
         double qq = Q[a * nshell + b] * Q[c * nshell + d];
         if (qq < tau) continue;

@@ -109,6 +109,22 @@ def jk(sh, D, tau=0.0, shard=0, nshards=1, pure=True, Q=None):
     return J, K
 
 
+def jk_qsample(sh, D, tau, shard, nshards, pure=True, Q=None):
+    """J/K over the canonical quartets (P, R) with (P(P+1)/2 + R) % nshards == shard (orc_jk_qsample): a
+    uniform 1/nshards sample of every class for timing the oracle on large builds; shards sum to jk()."""
+    keep, args = _basis_args(sh, pure)
+    N = sh.nbf(pure)
+    D = np.ascontiguousarray(D, dtype=np.float64)
+    J = np.zeros((N, N)); K = np.zeros((N, N))
+    Qp = None
+    if Q is not None:
+        Q = np.ascontiguousarray(Q, dtype=np.float64)
+        Qp = _d(Q)
+    _check(_get().orc_jk_qsample(*args, _d(D), ctypes.c_double(tau), ctypes.c_longlong(shard),
+                                 ctypes.c_longlong(nshards), Qp, _d(J), _d(K)), "jk_qsample")
+    return J, K
+
+
 def jk_dw(sh, D, tau, tau_dw, pure=True, Q=None):
     """J/K with the Schwarz rule at tau plus density-weighted screening at tau_dw (orc_jk_dw)."""
     keep, args = _basis_args(sh, pure)

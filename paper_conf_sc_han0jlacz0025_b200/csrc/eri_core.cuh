@@ -318,21 +318,21 @@ __device__ __forceinline__ void dmma884(double& c0, double& c1, double a, double
                : "d"(a), "d"(b));
 }
 
-// GEMM1 k-loop of one R row (Eq. 7a): t1[mc][nt] += E~_ab[row chunk ch][p] [p|q] with the B fragment
-// gathered from the R row through htab (a6)
+// GEMM1 k-loop of one R row (Eq. 7a): t1[mc][nt] += E~_ab[row chunk ch][p] [p|q]; the A fragments come
+// from the fragment-order copy EA = EbraD + ij * frag_a_doubles (one coalesced warp load each), the B
+// fragment is gathered from the R row through htab (a6)
 template <class C>
-__device__ __forceinline__ void gemm1_row(double (&t1)[C::MC][C::NT1][2], const double* __restrict__ E,
+__device__ __forceinline__ void gemm1_row(double (&t1)[C::MC][C::NT1][2], const double* __restrict__ EA,
                                           const double* __restrict__ Rr, const uint16_t* __restrict__ htab, int ch,
-                                          int g, int t) {
+                                          int lane) {
+  const int g = lane >> 2, t = lane & 3;
 #pragma unroll
   for (int ks = 0; ks < C::KS1; ++ks) {
     const int pc = 4 * ks + t;
     double a[C::MC];
 #pragma unroll
-    for (int mc = 0; mc < C::MC; ++mc) {
-      const int row = 8 * (ch * C::MC + mc) + g;
-      a[mc] = (row < C::NAB && pc < C::NHAB) ? __ldg(E + row * C::NHAB + pc) : 0.0;
-    }
+    for (int mc = 0; mc < C::MC; ++mc)
+      a[mc] = (ch * C::MC + mc < C::MT) ? __ldg(EA + ((ch * C::MC + mc) * C::KS1 + ks) * 32 + lane) : 0.0;
 #pragma unroll
     for (int nt = 0; nt < C::NT1; ++nt) {
       const int qc = 8 * nt + g;
@@ -345,24 +345,26 @@ __device__ __forceinline__ void gemm1_row(double (&t1)[C::MC][C::NT1][2], const 
 }
 
 // GEMM2 (Eq. 7b / Eq. 11) chained in registers: k-step (nt, e) takes q = 8 nt + 2 t + e from the
-// GEMM1 accumulator of lane (g, t)
+// GEMM1 accumulator of lane (g, t); both B fragments of (nt, e = 0, 1) come with one 128-bit load from
+// the fragment-order copy EB = EketD + kl * frag_b_doubles
 template <class C>
 __device__ __forceinline__ void gemm2_chain(double (&c2)[C::MC][C::NT2][2], const double (&t1)[C::MC][C::NT1][2],
-                                            const double* __restrict__ Ek, int ch, int g, int t) {
+                                            const double* __restrict__ EB, int ch, int lane) {
 #pragma unroll
-  for (int nt = 0; nt < C::NT1; ++nt)
+  for (int nt = 0; nt < C::NT1; ++nt) {
+    double2 b[C::NT2];
 #pragma unroll
-    for (int e = 0; e < 2; ++e) {
-      const int qq = 8 * nt + 2 * t + e;
+    for (int n2 = 0; n2 < C::NT2; ++n2) b[n2] = __ldg(reinterpret_cast<const double2*>(EB) + (nt * C::NT2 + n2) * 32 + lane);
+    // k-step e = 0 over every (mc, n2) accumulator, then e = 1: consecutive DMMAs stay independent
 #pragma unroll
-      for (int n2 = 0; n2 < C::NT2; ++n2) {
-        const int cd = 8 * n2 + g;
-        const double b = (qq < C::NHCD && cd < C::NCD) ? __ldg(Ek + qq * C::NCD + cd) : 0.0;
+    for (int e = 0; e < 2; ++e)
+#pragma unroll
+      for (int n2 = 0; n2 < C::NT2; ++n2)
 #pragma unroll
         for (int mc = 0; mc < C::MC; ++mc)
-          if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
-      }
-    }
+          if (ch * C::MC + mc < C::MT)
+            dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], e ? b[n2].y : b[n2].x);
+  }
 }
 
 template <int L>
@@ -404,7 +406,7 @@ __device__ void quartet_block_rb(const PairView& bra, int b0, int KAB, const Pai
     }
     __syncwarp();
     for (int k = 0; k < nk; ++k) {
-      const double* __restrict__ Ek = ket.Eket + (size_t)(kb + k) * (C::NHCD * C::NCD);
+      const double* __restrict__ EB = ket.EketD + (size_t)(kb + k) * frag_b_doubles(C::LC, C::LD);
       for (int ch = 0; ch < C::NCHUNK; ++ch) {
         double t1[C::MC][C::NT1][2];
 #pragma unroll
@@ -412,15 +414,15 @@ __device__ void quartet_block_rb(const PairView& bra, int b0, int KAB, const Pai
 #pragma unroll
           for (int nt = 0; nt < C::NT1; ++nt) t1[mc][nt][0] = t1[mc][nt][1] = 0.0;
         for (int il = 0; il < KAB; ++il)
-          gemm1_row<C>(t1, bra.Ebra + (size_t)(b0 + il) * (C::NAB * C::NHAB), Rbuf + (k * KAB + il) * RS, htab, ch,
-                       g, t);
+          gemm1_row<C>(t1, bra.EbraD + (size_t)(b0 + il) * frag_a_doubles(C::LA, C::LB), Rbuf + (k * KAB + il) * RS,
+                       htab, ch, lane);
         if constexpr (!ONECHUNK) {
 #pragma unroll
           for (int mc = 0; mc < C::MC; ++mc)
 #pragma unroll
             for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
         }
-        gemm2_chain<C>(c2, t1, Ek, ch, g, t);
+        gemm2_chain<C>(c2, t1, EB, ch, lane);
         if constexpr (!ONECHUNK) {
 #pragma unroll
           for (int mc = 0; mc < C::MC; ++mc)
@@ -482,7 +484,7 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
   for (int kl = k0; kl < k1; ++kl) {
     double q, Qx, Qy, Qz;
     load_pdat(ket.pdat, kl, q, Qx, Qy, Qz);
-    const double* __restrict__ Ek = ket.Eket + (size_t)kl * (C::NHCD * C::NCD);
+    const double* __restrict__ EB = ket.EketD + (size_t)kl * frag_b_doubles(C::LC, C::LD);
     // single row chunk and one R row: stream the bra primitives through it, GEMM2 once per ket primitive
     constexpr bool STREAM = C::NCHUNK == 1 && KR == 1;
     double t1s[C::MC][C::NT1][2];
@@ -508,28 +510,9 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
             t1[mc][nt][0] = STREAM ? t1s[mc][nt][0] : 0.0;
             t1[mc][nt][1] = STREAM ? t1s[mc][nt][1] : 0.0;
           }
-        for (int il = 0; il < ign; ++il) {
-          const double* __restrict__ E = bra.Ebra + (size_t)(ig0 + il) * (C::NAB * C::NHAB);
-          const double* __restrict__ Rr = Rbuf + il * NH;
-#pragma unroll
-          for (int ks = 0; ks < C::KS1; ++ks) {
-            const int pc = 4 * ks + t;
-            double a[C::MC];
-#pragma unroll
-            for (int mc = 0; mc < C::MC; ++mc) {
-              const int row = 8 * (ch * C::MC + mc) + g;
-              a[mc] = (row < C::NAB && pc < C::NHAB) ? __ldg(E + row * C::NHAB + pc) : 0.0;
-            }
-#pragma unroll
-            for (int nt = 0; nt < C::NT1; ++nt) {
-              const int qc = 8 * nt + g;
-              const double b = (pc < C::NHAB && qc < C::NHCD) ? Rr[htab[pc * C::NHCD + qc]] : 0.0;
-#pragma unroll
-              for (int mc = 0; mc < C::MC; ++mc)
-                if (ch * C::MC + mc < C::MT) dmma884(t1[mc][nt][0], t1[mc][nt][1], a[mc], b);
-            }
-          }
-        }
+        for (int il = 0; il < ign; ++il)
+          gemm1_row<C>(t1, bra.EbraD + (size_t)(ig0 + il) * frag_a_doubles(C::LA, C::LB), Rbuf + il * NH, htab, ch,
+                       lane);
         if constexpr (STREAM) {
           // keep accumulating over the next bra primitives; GEMM2 after the last one
 #pragma unroll
@@ -547,21 +530,7 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
 #pragma unroll
             for (int n2 = 0; n2 < C::NT2; ++n2) c2[mc][n2][0] = c2[mc][n2][1] = 0.0;
         }
-        // GEMM2: k-step (nt, e) takes q = 8 nt + 2 t + e from the GEMM1 accumulator of lane (g, t)
-#pragma unroll
-        for (int nt = 0; nt < C::NT1; ++nt)
-#pragma unroll
-          for (int e = 0; e < 2; ++e) {
-            const int qq = 8 * nt + 2 * t + e;
-#pragma unroll
-            for (int n2 = 0; n2 < C::NT2; ++n2) {
-              const int cd = 8 * n2 + g;
-              const double b = (qq < C::NHCD && cd < C::NCD) ? __ldg(Ek + qq * C::NCD + cd) : 0.0;
-#pragma unroll
-              for (int mc = 0; mc < C::MC; ++mc)
-                if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
-            }
-          }
+        gemm2_chain<C>(c2, t1, EB, ch, lane);
         if constexpr (!ONECHUNK) {
 #pragma unroll
           for (int mc = 0; mc < C::MC; ++mc)
@@ -592,17 +561,19 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
 }
 
 // Orientation of an R x C block of J/K updates in the non-symmetrised accumulators (J = Jacc + Jacc^T,
-// K = Kacc + Kacc^T at the end of the build, so element (r, c) may go to (r, c) or (c, r)): the
-// orientation with the longer contiguous runs (R > C: transposed).  blk_rc maps the y-th element of the
-// block to (r, c) so that consecutive y are adjacent in memory; blk_dst is its accumulator offset.
-template <int R, int C>
+// K = Kacc + Kacc^T at the end of the build, so element (r, c) may go to (r, c) or (c, r)).  blk_rc maps
+// the y-th element of the block to (r, c) so that consecutive y are adjacent in memory; blk_dst is its
+// accumulator offset.  FLIP allows the transposed orientation when it gives longer runs (R > C); the
+// K blocks never flip: their rows are the task's bra shells, and keeping every update of a task in
+// those few rows is what keeps them L2-resident (flipped, the (dp|pp) slab kernel ran 16 % slower).
+template <int R, int C, bool FLIP = false>
 __device__ __forceinline__ void blk_rc(int y, int& r, int& c) {
-  if constexpr (R > C) { c = y / R; r = y % R; }
+  if constexpr (FLIP && R > C) { c = y / R; r = y % R; }
   else { r = y / C; c = y % C; }
 }
-template <int R, int C>
+template <int R, int C, bool FLIP = false>
 __device__ __forceinline__ size_t blk_dst(int row, int col, int nbf) {
-  if constexpr (R > C) return (size_t)col * nbf + row;
+  if constexpr (FLIP && R > C) return (size_t)col * nbf + row;
   else return (size_t)row * nbf + col;
 }
 
@@ -717,11 +688,9 @@ __device__ void digest(const double* __restrict__ V, double deg, int oa, int ob,
   __syncwarp();
   // 4. K_ac[a][c] = sum_d P_ac[a][c,d] | K_ad[a][d] = sum_c P_ad[a][c,d] |
   //    K_bc[b][c] = sum_d P_bc[b][c,d] | K_bd[b][d] = sum_c P_bd[b][c,d]
-  //    Each block goes to the accumulator in the orientation whose rows are longer (K = Kacc + Kacc^T
-  //    at the end, so either triangle is exact) and consecutive lanes take consecutive columns: one RED
-  //    instruction then covers runs of up to 7 adjacent doubles, and the L2 atomic units work per
-  //    32-byte sector (measured 1.65e11 sectors/s, 4.2e11 doubles/s with 4 doubles per sector,
-  //    tools/atomics_bench.cu)
+  //    Consecutive lanes take adjacent columns of a bra row, so one RED instruction covers runs of NC
+  //    or ND adjacent doubles (the L2 atomic units work per 32-byte sector: measured 1.65e11 sectors/s,
+  //    4.2e11 doubles/s with 4 doubles per sector, tools/atomics_bench.cu)
   constexpr int N1 = NA * NC, N2 = N1 + NA * ND, N3 = N2 + NB * NC, N4 = N3 + NB * ND;
   constexpr int NMX = NC > ND ? NC : ND;
   for (int x = lane; x < N4; x += 32) {

@@ -17,9 +17,6 @@
 
 namespace mako {
 
-#ifndef MAKO_KF_EKREG
-#define MAKO_KF_EKREG 0
-#endif
 template <int X, int Y>
 struct KfCfg {
   using C = ClsXY<X, Y>;
@@ -151,11 +148,6 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
         double Rr[nH(L)];
         r_regs<L>(p, Px, Py, Pz, q, Qx, Qy, Qz, a.boys, Rr);
         const double* __restrict__ ek = a.ket.Eket + (size_t)kl * (NHCD * NCD);
-        // small ket E~ (ss, ps kets): the whole matrix with 256-bit loads up front (fewer L1 requests;
-        // the kernel is L1-bound, profiles/README.md); larger ones row by row
-        constexpr bool EK_REG = MAKO_KF_EKREG && NHCD * NCD <= 16;
-        double Ekr[EK_REG ? NHCD : 1][EK_REG ? NCD : 1];
-        if constexpr (EK_REG) load_mat<NHCD, NCD>(ek, Ekr);
         static_for<0, LPK>([&](auto hc) {
           constexpr int H = decltype(hc)::value;
           constexpr int p0 = H * PP, p1 = (p0 + PP < NHAB) ? p0 + PP : NHAB;
@@ -164,10 +156,7 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
               constexpr int qq = decltype(qc)::value;
               double e[NCD];
 #pragma unroll
-              for (int j = 0; j < NCD; ++j) {
-                if constexpr (EK_REG) e[j] = Ekr[qq][j];
-                else e[j] = __ldg(ek + qq * NCD + j);
-              }
+              for (int j = 0; j < NCD; ++j) e[j] = __ldg(ek + qq * NCD + j);
               static_for<p0, p1>([&](auto pc) {
                 constexpr int pp = decltype(pc)::value;
                 constexpr int hs = h_sum(pp, qq);
@@ -188,16 +177,13 @@ __device__ __forceinline__ void kf_body(const JKArgs& a) {
       }
       __syncwarp();
       // ---- DMMA stage: V[ab][(k,cd)] += E~_ab^{ij} W ----
-      const double* __restrict__ E = a.bra.Ebra + (size_t)ij * (NAB * NHAB);
+      const double* __restrict__ EA = a.bra.EbraD + (size_t)ij * frag_a_doubles(C::LA, C::LB);  // A fragments
 #pragma unroll
       for (int ks = 0; ks < KS1; ++ks) {
         const int pc = 4 * ks + t;
         double af[MT];
 #pragma unroll
-        for (int m = 0; m < MT; ++m) {
-          const int row = 8 * m + g;
-          af[m] = (row < NAB && pc < NHAB) ? __ldg(E + row * NHAB + pc) : 0.0;
-        }
+        for (int m = 0; m < MT; ++m) af[m] = __ldg(EA + (m * KS1 + ks) * 32 + lane);
 #pragma unroll
         for (int n = 0; n < NTV; ++n) {
           const double b = Ws[pc * WS + 8 * n + g];

@@ -174,16 +174,12 @@ __global__ void __launch_bounds__(128) slab_jk_kernel(JKArgs a) {
         __syncwarp();
         // GEMM1 (blocked layout): T1[ab][(s,q)] += E~_ab^{ij} R^{(ij,s)}_{p+q}
         for (int ijl = 0; ijl < ijn; ++ijl) {
-          const double* __restrict__ E = a.bra.Ebra + (size_t)(b0 + ij0 + ijl) * (NAB * NHAB);
+          const double* __restrict__ EA = a.bra.EbraD + (size_t)(b0 + ij0 + ijl) * frag_a_doubles(C::LA, C::LB);
 #pragma unroll
           for (int ks = 0; ks < KS1; ++ks) {
-            const int pc = 4 * ks + t;
             double af[MT];
 #pragma unroll
-            for (int m = 0; m < MT; ++m) {
-              const int row = 8 * m + g;
-              af[m] = (row < NAB && pc < NHAB) ? __ldg(E + row * NHAB + pc) : 0.0;
-            }
+            for (int m = 0; m < MT; ++m) af[m] = __ldg(EA + (m * KS1 + ks) * 32 + lane);
 #pragma unroll
             for (int n = 0; n < NT1B; ++n) {
               const int h = hofs[(ks * NT1B + n) * 32 + lane];

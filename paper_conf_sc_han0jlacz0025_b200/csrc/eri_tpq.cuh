@@ -171,20 +171,21 @@ __device__ __forceinline__ void sh_add(double* p, double v) { atomicAdd(p, v); }
 
 // Sector-grouped digestion of one R x C block per lane (lane = ket) of the lane-per-ket kernel: the
 // lanes' block values go through warp shared memory so that each RED instruction covers, for ~32/run
-// kets, a run of adjacent doubles (the block orientation with the longer runs, blk_rc / blk_dst in
-// eri_core.cuh): the L2 atomic units are bound per 32-byte sector, not per double (1.65e11 sectors/s
-// measured, tools/atomics_bench.cu), and the direct per-lane atomics hit one sector per double.
+// kets, a run of adjacent doubles (blk_rc / blk_dst in eri_core.cuh; K blocks stay in the bra rows):
+// the L2 atomic units are bound per 32-byte sector, not per double (1.65e11 sectors/s measured,
+// tools/atomics_bench.cu), and the direct per-lane atomics hit one sector per double.  Used for p kets
+// (runs of 3 adjacent columns); for s kets every run is one double.
 #ifndef MAKO_TPQ_STAGE
-#define MAKO_TPQ_STAGE 1
+#define MAKO_TPQ_STAGE 0  // measured: 11.37 s/build without, 11.51 s with (the SMEM round trip costs more)
 #endif
-template <int R, int CC, class F>
+template <int R, int CC, bool FLIP, class F>
 __device__ __forceinline__ void staged_red(double* __restrict__ out, double* __restrict__ stage, int lane, bool active,
                                            int orow, int ocol, int nbf, F&& val) {
   constexpr int E = R * CC;
 #pragma unroll
   for (int y = 0; y < E; ++y) {
     int r, c;
-    blk_rc<R, CC>(y, r, c);
+    blk_rc<R, CC, FLIP>(y, r, c);
     stage[lane * E + y] = active ? val(r, c) : 0.0;
   }
   __syncwarp();
@@ -194,8 +195,8 @@ __device__ __forceinline__ void staged_red(double* __restrict__ out, double* __r
     const int orw = __shfl_sync(0xffffffffu, orow, ket), ocl = __shfl_sync(0xffffffffu, ocol, ket);
     const double v = stage[idx];
     int r, c;
-    blk_rc<R, CC>(y, r, c);
-    if (v != 0.0) atomicAdd(out + blk_dst<R, CC>(orw + r, ocl + c, nbf), v);
+    blk_rc<R, CC, FLIP>(y, r, c);
+    if (v != 0.0) atomicAdd(out + blk_dst<R, CC, FLIP>(orw + r, ocl + c, nbf), v);
   }
   __syncwarp();
 }
@@ -335,16 +336,16 @@ __device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1,
         else atomicAdd(a.J + (oa + i / NB) * n + ob + i % NB, 2.0 * s);
       }
     }
-    if constexpr (!STRIP && MAKO_TPQ_STAGE) {
+    if constexpr (!STRIP && MAKO_TPQ_STAGE && NC > 1) {
       const double* __restrict__ Db = Dm;
       // J_cd ; K_ac += v D_bd ; K_ad += v D_bc ; K_bc += v D_ad ; K_bd += v D_ac (deg = 0 on idle lanes)
-      staged_red<NC, ND>(a.J, stage, lane, active, oc, od, a.nbf, [&](int k, int l) {
+      staged_red<NC, ND, true>(a.J, stage, lane, active, oc, od, a.nbf, [&](int k, int l) {
         double s = 0.0;
 #pragma unroll
         for (int ij = 0; ij < NAB; ++ij) s = fma(V[ij][k * ND + l], __ldg(Db + (oa + ij / NB) * n + ob + ij % NB), s);
         return 2.0 * deg * s;
       });
-      staged_red<NA, NC>(a.K, stage, lane, active, oa, oc, a.nbf, [&](int i, int k) {
+      staged_red<NA, NC, false>(a.K, stage, lane, active, oa, oc, a.nbf, [&](int i, int k) {
         double s = 0.0;
 #pragma unroll
         for (int j = 0; j < NB; ++j)
@@ -352,7 +353,7 @@ __device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1,
           for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Db + (ob + j) * n + od + l), s);
         return deg * s;
       });
-      staged_red<NA, ND>(a.K, stage, lane, active, oa, od, a.nbf, [&](int i, int l) {
+      staged_red<NA, ND, false>(a.K, stage, lane, active, oa, od, a.nbf, [&](int i, int l) {
         double s = 0.0;
 #pragma unroll
         for (int j = 0; j < NB; ++j)
@@ -360,7 +361,7 @@ __device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1,
           for (int k = 0; k < NC; ++k) s = fma(V[i * NB + j][k * ND + l], __ldg(Db + (ob + j) * n + oc + k), s);
         return deg * s;
       });
-      staged_red<NB, NC>(a.K, stage, lane, active, ob, oc, a.nbf, [&](int j, int k) {
+      staged_red<NB, NC, false>(a.K, stage, lane, active, ob, oc, a.nbf, [&](int j, int k) {
         double s = 0.0;
 #pragma unroll
         for (int i = 0; i < NA; ++i)
@@ -368,7 +369,7 @@ __device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1,
           for (int l = 0; l < ND; ++l) s = fma(V[i * NB + j][k * ND + l], __ldg(Db + (oa + i) * n + od + l), s);
         return deg * s;
       });
-      staged_red<NB, ND>(a.K, stage, lane, active, ob, od, a.nbf, [&](int j, int l) {
+      staged_red<NB, ND, false>(a.K, stage, lane, active, ob, od, a.nbf, [&](int j, int l) {
         double s = 0.0;
 #pragma unroll
         for (int i = 0; i < NA; ++i)

@@ -76,6 +76,9 @@ MK_HD constexpr int class_kt(int X, int Y) { return use_tpq(X, Y) ? 32 : 16; }
 MK_HD constexpr int lowp_a_floats(int la, int lb) {
   return ((nsph(la) * nsph(lb) + 15) / 16) * ((nH(la + lb) + 7) / 8) * 128;
 }
+// FP64 fragment-order copies (m8n8k4): doubles per primitive pair
+MK_HD constexpr int frag_a_doubles(int la, int lb) { return ((nsph(la) * nsph(lb) + 7) / 8) * ((nH(la + lb) + 3) / 4) * 32; }
+MK_HD constexpr int frag_b_doubles(int la, int lb) { return ((nH(la + lb) + 7) / 8) * ((nsph(la) * nsph(lb) + 7) / 8) * 64; }
 MK_HD constexpr int lowp_b_floats(int la, int lb) {
   return ((nH(la + lb) + 7) / 8) * ((nsph(la) * nsph(lb) + 7) / 8) * 64;
 }
@@ -177,6 +180,11 @@ struct PairView {
   const double* pdat;    // [nprim][4]: p, Px, Py, Pz
   const double* Ebra;    // [nprim][nab][nHab]  E~ with spherical transform, coefficients, 1/p folded
   const double* Eket;    // [nprim][nHab][nab]  (-1)^{|q|} E~^T
+  // FP64 copies in mma.m8n8k4 fragment order (one coalesced warp load per fragment; pairs.cu
+  // build_frag_kernel): GEMM1 A fragments [nprim][MT8][KS4][32 lanes] of E~ and GEMM2 B fragments
+  // [nprim][NT8(q)][NT8(cd)][32 lanes][2] of (-1)^{|q|} E~^T
+  const double* EbraD;
+  const double* EketD;
   // reduced-precision tier (null until first requested): TF32 copies in mma fragment order
   const float* EbraF;    // [nprim][MT16][KS8][32 lanes][4]  GEMM1 A fragments of E~
   const float* EketF;    // [nprim][NT8(q)][NT8(cd)][32 lanes][2]  GEMM2 B fragments of (-1)^{|q|} E~^T

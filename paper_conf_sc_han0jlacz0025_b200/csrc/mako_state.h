@@ -45,6 +45,7 @@ struct PairBucket {
   std::vector<int> poff;           // [n+1]
   std::vector<int> seg;            // [NKGROUP+1] K-group segment starts (screened sets only)
   DevBuf d_shA, d_shB, d_Q, d_poff, d_pdat, d_Ebra, d_Eket;
+  DevBuf d_EbraD, d_EketD;         // FP64 m8n8k4 fragment-order copies (DMMA operand loads)
   DevBuf d_EbraF, d_EketF;         // TF32 fragment-order copies (reduced-precision tier, built on demand)
   int n() const { return (int)shA.size(); }
   PairView view() const;

@@ -135,9 +135,40 @@ PairView PairBucket::view() const {
   v.pdat = d_pdat.as<double>();
   v.Ebra = d_Ebra.as<double>();
   v.Eket = d_Eket.as<double>();
+  v.EbraD = d_EbraD.as<double>();
+  v.EketD = d_EketD.as<double>();
   v.EbraF = d_EbraF.as<float>();
   v.EketF = d_EketF.as<float>();
   return v;
+}
+
+// FP64 copies of E~ in mma.m8n8k4 fragment order, zero-padded: A fragments of GEMM1 (lane (g,t):
+// E~[8m+g][4k+t]) and B fragment pairs of GEMM2 (lane (g,t): Ek[8n+2t][8j+g], Ek[8n+2t+1][8j+g]).
+// One thread per output double.
+__global__ void build_frag_kernel(int nab, int nh, long long total_a, long long total_b, const double* __restrict__ Ebra,
+                                  const double* __restrict__ Eket, double* __restrict__ EbraD,
+                                  double* __restrict__ EketD) {
+  const int MT = (nab + 7) / 8, KS = (nh + 3) / 4, NQ = (nh + 7) / 8, NC = (nab + 7) / 8;
+  const int AF = MT * KS * 32, BF = NQ * NC * 64;
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < total_a + total_b;
+       x += (long long)gridDim.x * blockDim.x) {
+    double v = 0.0;
+    if (x < total_a) {
+      const long long id = x / AF;
+      const int r = (int)(x % AF), mk = r / 32, lane = r % 32;
+      const int m = mk / KS, k = mk % KS, g = lane >> 2, t = lane & 3;
+      const int row = 8 * m + g, col = 4 * k + t;
+      if (row < nab && col < nh) v = Ebra[(size_t)id * nab * nh + (size_t)row * nh + col];
+      EbraD[x] = v;
+    } else {
+      const long long y = x - total_a, id = y / BF;
+      const int r = (int)(y % BF), nj = r / 64, lane = (r % 64) / 2, e = r % 2;
+      const int n = nj / NC, j = nj % NC, g = lane >> 2, t = lane & 3;
+      const int q = 8 * n + 2 * t + e, cd = 8 * j + g;
+      if (q < nh && cd < nab) v = Eket[(size_t)id * nab * nh + (size_t)q * nab + cd];
+      EketD[y] = v;
+    }
+  }
 }
 
 // Build device pair data for the given per-bucket shell lists (A has the higher l).
@@ -189,6 +220,17 @@ mako_status build_pair_set(const mako_basis_s* B, const std::vector<int> (&A)[NB
                                         pb.d_Eket.as<double>());
       if ((st = cuda_check(cudaGetLastError(), "build_E_kernel"))) return st;
     }
+    {
+      const long long ta = (long long)std::max(np, 1) * frag_a_doubles(pb.la, pb.lb);
+      const long long tb = (long long)std::max(np, 1) * frag_b_doubles(pb.la, pb.lb);
+      if ((st = pb.d_EbraD.alloc(sizeof(double) * ta)) || (st = pb.d_EketD.alloc(sizeof(double) * tb))) return st;
+      if (np > 0) {
+        build_frag_kernel<<<1184, 256, 0, s>>>(nsph(pb.la) * nsph(pb.lb), nH(pb.la + pb.lb), ta, tb,
+                                               pb.d_Ebra.as<double>(), pb.d_Eket.as<double>(), pb.d_EbraD.as<double>(),
+                                               pb.d_EketD.as<double>());
+        if ((st = cuda_check(cudaGetLastError(), "build_frag_kernel"))) return st;
+      }
+    }
     // temporaries are freed at scope exit: make sure the kernel is done with them
     if ((st = cuda_check(cudaStreamSynchronize(s), "build_pair_set sync"))) return st;
   }
@@ -234,11 +276,14 @@ mako_status ensure_lowp(PairSet& set, void* stream) {
   for (int b = 0; b < NBUCKET; ++b) {
     PairBucket& pb = set.b[b];
     if (pb.d_EbraF.p) continue;
+    // an empty bucket keeps a one-element allocation and no kernel (its E~ was never written)
     const long long np = std::max(pb.poff.empty() ? 0 : pb.poff.back(), 1);
+    const bool empty = pb.poff.empty() || pb.poff.back() == 0;
     const int nab = nsph(pb.la) * nsph(pb.lb), nh = nH(pb.la + pb.lb);
     const long long ta = np * lowp_a_floats(pb.la, pb.lb), tb = np * lowp_b_floats(pb.la, pb.lb);
     mako_status st;
     if ((st = pb.d_EbraF.alloc(sizeof(float) * ta)) || (st = pb.d_EketF.alloc(sizeof(float) * tb))) return st;
+    if (empty) continue;
     build_lowp_kernel<<<1184, 256, 0, s>>>(nab, nh, ta, tb, pb.d_Ebra.as<double>(), pb.d_Eket.as<double>(),
                                           pb.d_EbraF.as<float>(), pb.d_EketF.as<float>());
     if ((st = cuda_check(cudaGetLastError(), "build_lowp_kernel"))) return st;
@@ -334,6 +379,8 @@ extern "C" mako_status mako_shellpairs_screen(mako_basis basis, double thresh, v
     for (int b = 0; b < NBUCKET; ++b) {  // free candidate device memory before the rebuild
       cand.b[b].d_Ebra.release();
       cand.b[b].d_Eket.release();
+      cand.b[b].d_EbraD.release();
+      cand.b[b].d_EketD.release();
     }
     if ((st = build_pair_set(basis, A2, B2, P->set, cuda_stream))) return st;
     cudaStream_t s = (cudaStream_t)cuda_stream;

@@ -110,3 +110,28 @@ def test_schwarz_screening_error_bound():
     bound = 4 * tau * np.abs(D).max() * 49 * max(ndrop, 1)
     assert ndrop > 0
     assert np.abs(J1 - J0).max() <= bound and np.abs(K1 - K0).max() <= bound
+
+
+def test_quartet_sample_shards_sum_to_full_build():
+    """orc_jk_qsample (the timing sample of bench.py's cpu_baseline / reference arm): the quartet shards
+    (canonical quartet index % n == shard) partition the build exactly, for n below and above the number
+    of canonical quartets."""
+    import mako_inputs as mi
+    m, b = mi.config_molecule("benzene-def2svp")
+    sh = mi.shells_for(m, b).subset(list(range(14)))
+    D = mi.synthetic_density(sh.nbf(), 6, seed=2)
+    J0, K0 = oracle.jk(sh, D, 1e-12)
+    for n in (5, 13, 20000):
+        Js, Ks = np.zeros_like(J0), np.zeros_like(K0)
+        for s in range(n if n < 100 else 0):
+            j, k = oracle.jk_qsample(sh, D, 1e-12, s, n)
+            Js += j
+            Ks += k
+        if n >= 100:  # sample a few shards only: a non-matching shard is empty, a matching one is one quartet
+            nq = sh.nshell * (sh.nshell + 1) // 2
+            nq = nq * (nq + 1) // 2
+            empty, _ = oracle.jk_qsample(sh, D, 1e-12, nq, nq + 1)
+            assert not empty.any()
+            continue
+        assert np.abs(Js - J0).max() <= 1e-12 * np.abs(J0).max()
+        assert np.abs(Ks - K0).max() <= 1e-12 * np.abs(K0).max()

@@ -1,0 +1,32 @@
+"""Per-class A/B table of round-2 kernel experiments (bench.py --class-times lines under profiles/ab_r02/):
+    python tools/ab_table.py > profiles/bench_r02_ab.md"""
+import json
+import os
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+RUNS = [("r2b_nostrip", "round-1 kernels (interleaved shards)"), ("r2b_strip", "+ K-row strips (lane-per-ket)"),
+        ("r2b_swap", "+ strips, 25 classes transposed"), ("r2c_rb", "+ strips, batched R (L <= 7)"),
+        ("r2d_rbswap", "+ strips, batched R + transposed"), ("r2e_rb2", "no strips, batched R (L <= 6) incl. (pp|pp) ... (dp|ds) moved to family 4"),
+        ("r2e_rb2s", "r2e_rb2 + (ds|pp) (dp|pp) (dp|ds) transposed"), ("r2f_main", "picks + flipped K atomics + staged lane-per-ket atomics"),
+        ("r2g_main", "picks + bra-row K atomics + staged lane-per-ket atomics"), ("r2i_nostage", "r2g_main without staging"),
+        ("r2i_main", "r2g_main + fragment-order E~ (DMMA operands)")]
+d = {}
+for name, _ in RUNS:
+    p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
+    if os.path.exists(p):
+        d[name] = json.loads(open(p).read())
+names = [n for n, _ in RUNS if n in d]
+print("# Round-2 kernel experiments, per class (valinomycin-sized def2-TZVP build, ms per class kernel)\n")
+print("Each column is one `bench.py --class-times` run on a B200 (`tools/exp/r2_*.sh`); the build total is the")
+print("first row.  Lower is better.\n")
+for n, desc in RUNS:
+    if n in d:
+        print(f"- `{n}`: {desc}")
+print()
+print("| class | " + " | ".join(names) + " |")
+print("|---|" + "---|" * len(names))
+print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names) + " |")
+classes = list(d[names[0]]["class_ms"])
+classes.sort(key=lambda k: -d[names[0]]["class_ms"][k][0])
+for k in classes:
+    print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names) + " |")

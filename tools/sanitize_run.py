@@ -1,5 +1,6 @@
 """Small J/K workloads that reach every kernel family, for compute-sanitizer:
-    compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize_run.py
+    compute-sanitizer --tool {memcheck,synccheck,initcheck} python tools/sanitize_run.py
+    compute-sanitizer --tool racecheck python tools/sanitize_run.py small   (racecheck is ~1000x slower)
 benzene def2-SVP (plain, density-screened, mixed-precision tiers), a contracted s/p/d/f basis on 3 centres
 (every l <= 3 class, all five families incl. the transposed ones), a 2-centre s..g basis (the l = 4
 classes), mako_eri_batch (store kernels, FP64 and TF32) and an accumulate build."""
@@ -44,14 +45,17 @@ def run(sh, Z, xyz, nocc, mixed=True):
     return B
 
 
-m, b = mi.config_molecule("benzene-def2svp")
-run(mi.shells_for(m, b), m.Z, m.xyz_bohr, m.nelec // 2)
-sh, Z, xyz = basis(3, 3, (1, 3), 0)
-B = run(sh, Z, xyz, 10)
+small = len(sys.argv) > 1 and sys.argv[1] == "small"  # racecheck: the 3-centre s/p/d/f basis only
+if not small:
+    m, b = mi.config_molecule("benzene-def2svp")
+    run(mi.shells_for(m, b), m.Z, m.xyz_bohr, m.nelec // 2)
+sh, Z, xyz = basis(3 if not small else 2, 3, (1, 3), 0)
+B = run(sh, Z, xyz, 10 if not small else 6)
 q = [[int(a), int(b_), int(c), int(d)] for a, b_, c, d in np.random.default_rng(0).integers(0, sh.nshell, (64, 4))]
 eri_batch(B, q)
 eri_batch(B, q, reduced=True)
-sh, Z, xyz = basis(2, 4, (1, 2), 3)
-run(sh, Z, xyz, 8, mixed=False)
+if not small:
+    sh, Z, xyz = basis(2, 4, (1, 2), 3)
+    run(sh, Z, xyz, 8, mixed=False)
 torch.cuda.synchronize()
 print("sanitize workload done")
