@@ -41,7 +41,7 @@ PRIM_EPS = 1e-18  # primitive-pair rule of include/mako.h (reading R7)
 
 
 def peaks():
-    p = os.path.join(ROOT, "profiles", "peaks_fp64_r01.json")
+    p = os.path.join(ROOT, "profiles", "peaks_fp64_r02.json")
     d = json.load(open(p))
     return d
 
@@ -416,8 +416,9 @@ def run_mako(args):
             "frac": achieved / pk["dmma_m16n8k4_tflops"], "traffic": traffic,
             "kernel": f"{FAMILY_KERNELS[int(class_family()[c])]}<{X},{Y}> class ({names[X]}|{names[Y]})",
             "share_of_step": float(cls_ms[c] / max(cls_ms.sum(), 1e-9)),
-            "peak_source": "FP64 DMMA mma.sync m16n8k4 loop measured on this pool's B200 "
-                           "(profiles/peaks_fp64_r01.json; MEASURED_PEAKS.json has no FP64 entry)",
+            "peak_source": "FP64 DMMA mma.sync m16n8k4 loop measured on this pool's B200 with the clock record "
+                           "(profiles/peaks_fp64_r02.json: 1965 MHz, no throttle reason; MEASURED_PEAKS.json "
+                           "has no FP64 entry)",
             "all_classes_achieved": value / world, "all_classes_frac": value / world / pk["dmma_m16n8k4_tflops"]}
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,

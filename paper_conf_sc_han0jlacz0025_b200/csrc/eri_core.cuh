@@ -57,7 +57,11 @@ struct Cls {
   // primitives) are computed lane-per-quartet in registers (r_regs) and stored at the odd stride RS
   static constexpr bool RBATCH = L <= 6 && in_list(kRBatchPick, bucket_of(LA, LB) * 100 + bucket_of(LC, LD));
   static constexpr int RB = 16, RS = NH | 1;
-  static constexpr int W_RCOOP = (KR + 1) * NH > RB * RS || !RBATCH ? (KR + 1) * NH : RB * RS;
+  static constexpr int W_RBAT = RBATCH ? RB * RS : 0;
+  static constexpr int W_RCOOP = (KR + 1) * NH > W_RBAT ? (KR + 1) * NH : W_RBAT;
+  // GEMM2 B operands from the fragment-order copy (default) or the row-major E~ (classes measured faster
+  // that way, MAKO_NOFRAGB_PICK; S6)
+  static constexpr bool FRAGB = !in_list(kNoFragBPick, bucket_of(LA, LB) * 100 + bucket_of(LC, LD));
   // KR result rows + 1 ping-pong scratch row; doubles as the digestion partial-sum scratch (Ps)
   static constexpr int W_R = (W_RCOOP > 2 * (NA + NB) * NCD) ? W_RCOOP : 2 * (NA + NB) * NCD;
   static constexpr int W_V = NAB * NCD; // (ab|cd) block
@@ -318,6 +322,17 @@ __device__ __forceinline__ void dmma884(double& c0, double& c1, double a, double
                : "d"(a), "d"(b));
 }
 
+// GEMM1 A operands from the fragment-order copy (MAKO_FRAG_A, default) or the row-major E~ (experiment
+// switch); the GEMM2 B operand choice is per class (Cls::FRAGB)
+#ifndef MAKO_FRAG_A
+#define MAKO_FRAG_A 1
+#endif
+template <class C>
+__device__ __forceinline__ const double* ebra_ptr(const PairView& bra, int ij) {
+  if constexpr (MAKO_FRAG_A) return bra.EbraD + (size_t)ij * frag_a_doubles(C::LA, C::LB);
+  else return bra.Ebra + (size_t)ij * (C::NAB * C::NHAB);
+}
+
 // GEMM1 k-loop of one R row (Eq. 7a): t1[mc][nt] += E~_ab[row chunk ch][p] [p|q]; the A fragments come
 // from the fragment-order copy EA = EbraD + ij * frag_a_doubles (one coalesced warp load each), the B
 // fragment is gathered from the R row through htab (a6)
@@ -331,8 +346,14 @@ __device__ __forceinline__ void gemm1_row(double (&t1)[C::MC][C::NT1][2], const 
     const int pc = 4 * ks + t;
     double a[C::MC];
 #pragma unroll
-    for (int mc = 0; mc < C::MC; ++mc)
-      a[mc] = (ch * C::MC + mc < C::MT) ? __ldg(EA + ((ch * C::MC + mc) * C::KS1 + ks) * 32 + lane) : 0.0;
+    for (int mc = 0; mc < C::MC; ++mc) {
+      if constexpr (MAKO_FRAG_A) {
+        a[mc] = (ch * C::MC + mc < C::MT) ? __ldg(EA + ((ch * C::MC + mc) * C::KS1 + ks) * 32 + lane) : 0.0;
+      } else {  // EA = row-major E~_ab of the primitive pair
+        const int row = 8 * (ch * C::MC + mc) + g;
+        a[mc] = (row < C::NAB && pc < C::NHAB) ? __ldg(EA + row * C::NHAB + pc) : 0.0;
+      }
+    }
 #pragma unroll
     for (int nt = 0; nt < C::NT1; ++nt) {
       const int qc = 8 * nt + g;
@@ -350,20 +371,37 @@ __device__ __forceinline__ void gemm1_row(double (&t1)[C::MC][C::NT1][2], const 
 template <class C>
 __device__ __forceinline__ void gemm2_chain(double (&c2)[C::MC][C::NT2][2], const double (&t1)[C::MC][C::NT1][2],
                                             const double* __restrict__ EB, int ch, int lane) {
+  if constexpr (C::FRAGB) {
 #pragma unroll
-  for (int nt = 0; nt < C::NT1; ++nt) {
-    double2 b[C::NT2];
+    for (int nt = 0; nt < C::NT1; ++nt) {
+      double2 b[C::NT2];
 #pragma unroll
-    for (int n2 = 0; n2 < C::NT2; ++n2) b[n2] = __ldg(reinterpret_cast<const double2*>(EB) + (nt * C::NT2 + n2) * 32 + lane);
-    // k-step e = 0 over every (mc, n2) accumulator, then e = 1: consecutive DMMAs stay independent
+      for (int n2 = 0; n2 < C::NT2; ++n2) b[n2] = __ldg(reinterpret_cast<const double2*>(EB) + (nt * C::NT2 + n2) * 32 + lane);
 #pragma unroll
-    for (int e = 0; e < 2; ++e)
+      for (int e = 0; e < 2; ++e)
 #pragma unroll
-      for (int n2 = 0; n2 < C::NT2; ++n2)
+        for (int n2 = 0; n2 < C::NT2; ++n2)
 #pragma unroll
-        for (int mc = 0; mc < C::MC; ++mc)
-          if (ch * C::MC + mc < C::MT)
-            dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], e ? b[n2].y : b[n2].x);
+          for (int mc = 0; mc < C::MC; ++mc)
+            if (ch * C::MC + mc < C::MT)
+              dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], e ? b[n2].y : b[n2].x);
+    }
+  } else {  // EB = row-major (-1)^{|q|} E~_cd^T of the primitive pair
+    const int g = lane >> 2, t = lane & 3;
+#pragma unroll
+    for (int nt = 0; nt < C::NT1; ++nt)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int qq = 8 * nt + 2 * t + e;
+#pragma unroll
+        for (int n2 = 0; n2 < C::NT2; ++n2) {
+          const int cd = 8 * n2 + g;
+          const double b = (qq < C::NHCD && cd < C::NCD) ? __ldg(EB + qq * C::NCD + cd) : 0.0;
+#pragma unroll
+          for (int mc = 0; mc < C::MC; ++mc)
+            if (ch * C::MC + mc < C::MT) dmma884(c2[mc][n2][0], c2[mc][n2][1], t1[mc][nt][e], b);
+        }
+      }
   }
 }
 
@@ -406,7 +444,8 @@ __device__ void quartet_block_rb(const PairView& bra, int b0, int KAB, const Pai
     }
     __syncwarp();
     for (int k = 0; k < nk; ++k) {
-      const double* __restrict__ EB = ket.EketD + (size_t)(kb + k) * frag_b_doubles(C::LC, C::LD);
+      const double* __restrict__ EB = C::FRAGB ? ket.EketD + (size_t)(kb + k) * frag_b_doubles(C::LC, C::LD)
+                                                  : ket.Eket + (size_t)(kb + k) * (C::NHCD * C::NCD);
       for (int ch = 0; ch < C::NCHUNK; ++ch) {
         double t1[C::MC][C::NT1][2];
 #pragma unroll
@@ -414,8 +453,7 @@ __device__ void quartet_block_rb(const PairView& bra, int b0, int KAB, const Pai
 #pragma unroll
           for (int nt = 0; nt < C::NT1; ++nt) t1[mc][nt][0] = t1[mc][nt][1] = 0.0;
         for (int il = 0; il < KAB; ++il)
-          gemm1_row<C>(t1, bra.EbraD + (size_t)(b0 + il) * frag_a_doubles(C::LA, C::LB), Rbuf + (k * KAB + il) * RS,
-                       htab, ch, lane);
+          gemm1_row<C>(t1, ebra_ptr<C>(bra, b0 + il), Rbuf + (k * KAB + il) * RS, htab, ch, lane);
         if constexpr (!ONECHUNK) {
 #pragma unroll
           for (int mc = 0; mc < C::MC; ++mc)
@@ -484,7 +522,8 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
   for (int kl = k0; kl < k1; ++kl) {
     double q, Qx, Qy, Qz;
     load_pdat(ket.pdat, kl, q, Qx, Qy, Qz);
-    const double* __restrict__ EB = ket.EketD + (size_t)kl * frag_b_doubles(C::LC, C::LD);
+    const double* __restrict__ EB = C::FRAGB ? ket.EketD + (size_t)kl * frag_b_doubles(C::LC, C::LD)
+                                                : ket.Eket + (size_t)kl * (C::NHCD * C::NCD);
     // single row chunk and one R row: stream the bra primitives through it, GEMM2 once per ket primitive
     constexpr bool STREAM = C::NCHUNK == 1 && KR == 1;
     double t1s[C::MC][C::NT1][2];
@@ -511,8 +550,7 @@ __device__ void quartet_block(const PairView& bra, int P, const PairView& ket, i
             t1[mc][nt][1] = STREAM ? t1s[mc][nt][1] : 0.0;
           }
         for (int il = 0; il < ign; ++il)
-          gemm1_row<C>(t1, bra.EbraD + (size_t)(ig0 + il) * frag_a_doubles(C::LA, C::LB), Rbuf + il * NH, htab, ch,
-                       lane);
+          gemm1_row<C>(t1, ebra_ptr<C>(bra, ig0 + il), Rbuf + il * NH, htab, ch, lane);
         if constexpr (STREAM) {
           // keep accumulating over the next bra primitives; GEMM2 after the last one
 #pragma unroll

@@ -125,6 +125,12 @@ constexpr int kJkSwapPick[] = {MAKO_JKSWAP_PICK};
 #define MAKO_RBATCH_PICK 207, 205, 602, 404, 202
 #endif
 constexpr int kRBatchPick[] = {MAKO_RBATCH_PICK};
+// warp-per-quartet classes (same codes) whose GEMM2 B operands are read from the row-major E~ rather
+// than the fragment-order copy (measured per class, profiles/bench_r02_ab.md)
+#ifndef MAKO_NOFRAGB_PICK
+#define MAKO_NOFRAGB_PICK 707, 602, 207, 109, 705, 309, 808, 205, 908, 905
+#endif
+constexpr int kNoFragBPick[] = {MAKO_NOFRAGB_PICK};
 constexpr int kJkCap4[] = {MAKO_JK_CAP4};
 constexpr int kKfCap3[] = {MAKO_KF_CAP3};
 template <int N>

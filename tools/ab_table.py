@@ -9,7 +9,10 @@ RUNS = [("r2b_nostrip", "round-1 kernels (interleaved shards)"), ("r2b_strip", "
         ("r2d_rbswap", "+ strips, batched R + transposed"), ("r2e_rb2", "no strips, batched R (L <= 6) incl. (pp|pp) ... (dp|ds) moved to family 4"),
         ("r2e_rb2s", "r2e_rb2 + (ds|pp) (dp|pp) (dp|ds) transposed"), ("r2f_main", "picks + flipped K atomics + staged lane-per-ket atomics"),
         ("r2g_main", "picks + bra-row K atomics + staged lane-per-ket atomics"), ("r2i_nostage", "r2g_main without staging"),
-        ("r2i_main", "r2g_main + fragment-order E~ (DMMA operands)")]
+        ("r2i_main", "r2g_main + fragment-order E~ (DMMA operands)"),
+        ("r2j_main", "r2i_main without staging, GEMM2 k-steps interleaved over accumulators"),
+        ("r2k_main", "r2j_main (repeat)"), ("r2k_nob", "r2k_main with row-major GEMM2 B operands"),
+        ("r2k_rbg", "r2k_main + batched R for L >= 7 with lane-group recursion (not kept)")]
 d = {}
 for name, _ in RUNS:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
