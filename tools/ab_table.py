@@ -13,8 +13,17 @@ RUNS = [("r2b_nostrip", "round-1 kernels (interleaved shards)"), ("r2b_strip", "
         ("r2j_main", "r2i_main without staging, GEMM2 k-steps interleaved over accumulators"),
         ("r2k_main", "r2j_main (repeat)"), ("r2k_nob", "r2k_main with row-major GEMM2 B operands"),
         ("r2k_rbg", "r2k_main + batched R for L >= 7 with lane-group recursion (not kept)")]
+# session 3: band/shell pair order with K_ac/K_bc run aggregation (S6, tools/exp/r2_band_order.patch)
+RUNS2 = [("r2n_pre", "fec4888 kernels (reference for this group)"),
+         ("r2m_allband_dmma", "all buckets in band order; run aggregation in every family (lane-per-ket, ket-first, DMMA)"),
+         ("r2m_q0_dmma", "the same kernels on the Q order (no runs)"),
+         ("r2o_allband", "all buckets in band order; aggregation in lane-per-ket + ket-first (values first, then the scan)"),
+         ("r2o_q0", "the same kernels on the Q order"),
+         ("r2p_allband_kfold", "all buckets in band order; aggregation in lane-per-ket only"),
+         ("r2q_tpqperm", "Q order storage, lane-per-ket classes walk a band permutation; aggregation in lane-per-ket"),
+         ("r2q_q0", "the same kernels on the Q order")]
 d = {}
-for name, _ in RUNS:
+for name, _ in RUNS + RUNS2:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
     if os.path.exists(p):
         d[name] = json.loads(open(p).read())
@@ -33,3 +42,16 @@ classes = list(d[names[0]]["class_ms"])
 classes.sort(key=lambda k: -d[names[0]]["class_ms"][k][0])
 for k in classes:
     print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names) + " |")
+
+names2 = [n for n, _ in RUNS2 if n in d]
+if names2:
+    print("\n## Band/shell pair order and K_ac/K_bc run aggregation (session 3; not kept)\n")
+    for n, desc in RUNS2:
+        if n in d:
+            print(f"- `{n}`: {desc}")
+    print()
+    print("| class | " + " | ".join(names2) + " |")
+    print("|---|" + "---|" * len(names2))
+    print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names2) + " |")
+    for k in classes:
+        print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names2) + " |")
