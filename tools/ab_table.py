@@ -22,8 +22,13 @@ RUNS2 = [("r2n_pre", "fec4888 kernels (reference for this group)"),
          ("r2p_allband_kfold", "all buckets in band order; aggregation in lane-per-ket only"),
          ("r2q_tpqperm", "Q order storage, lane-per-ket classes walk a band permutation; aggregation in lane-per-ket"),
          ("r2q_q0", "the same kernels on the Q order")]
+# session 3: super-batched R phase of the slot-batched kernel, and more classes on that kernel
+RUNS3 = [("r2r_pre", "fec4888 kernels (reference for this group)"),
+         ("r2r_superbatch", "slot-batched (dp|pp): R rows of RCAP / K_AB slots per R phase, one primitive quartet per lane (kept)"),
+         ("r2r_slab2", "+ (pp|pp) (fs|pp) (fs|dp) (fp|pp) on the slot-batched kernel"),
+         ("r2r_slab3", "ket-first classes (dp|ds) (fs|ds) (fp|ps) (fd|ps) (ds|pp) on the slot-batched kernel; (dp|ps) falls to lane-per-ket")]
 d = {}
-for name, _ in RUNS + RUNS2:
+for name, _ in RUNS + RUNS2 + RUNS3:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
     if os.path.exists(p):
         d[name] = json.loads(open(p).read())
@@ -55,3 +60,16 @@ if names2:
     print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names2) + " |")
     for k in classes:
         print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names2) + " |")
+
+names3 = [n for n, _ in RUNS3 if n in d]
+if names3:
+    print("\n## Slot-batched kernel with a super-batched R phase (session 3)\n")
+    for n, desc in RUNS3:
+        if n in d:
+            print(f"- `{n}`: {desc}")
+    print()
+    print("| class | " + " | ".join(names3) + " |")
+    print("|---|" + "---|" * len(names3))
+    print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names3) + " |")
+    for k in classes:
+        print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names3) + " |")
