@@ -93,10 +93,12 @@ MK_HD constexpr int kgroup(int K) {
                 : (K <= 6 ? 4 : (K <= 9 ? 5 : (K <= 12 ? 6 : (K <= 16 ? 7 : (K <= 24 ? 8 : (K <= 36 ? 9 : 10))))));
 }
 
-// Per-class kernel-family choices, measured on the bench workload (profiles/README.md).  Codes are
-// X * 100 + Y.  Overridable with -D for experiment builds (build.py --variant).
+// Per-class kernel-family choices, measured on the bench workload (profiles/README.md; re-selected in round 2
+// from all-on / all-off runs per family, profiles/bench_r02_ab.md: (dp|ps) left the ket-first kernel for the
+// lane-per-ket one, 531 -> 482 ms; (ff|dd) and (ff|fd) run transposed).  Codes are X * 100 + Y.  Overridable
+// with -D for experiment builds (build.py --variant).
 #ifndef MAKO_KF_PICK
-#define MAKO_KF_PICK 303, 401, 403, 501, 603, 701, 800, 801, 900, 700, 500
+#define MAKO_KF_PICK 303, 403, 501, 603, 701, 800, 801, 900, 700, 500
 #endif
 #ifndef MAKO_KFSWAP_PICK
 #define MAKO_KFSWAP_PICK 302
@@ -104,7 +106,7 @@ MK_HD constexpr int kgroup(int K) {
 // warp-per-quartet classes run transposed ((ab|cd) as (cd|ab): the ket side takes the inner, per
 // primitive-quartet GEMM1; S6), measured per class
 #ifndef MAKO_JKSWAP_PICK
-#define MAKO_JKSWAP_PICK 703, 803, 706, 503, 802, 806, 901, 804, 502, 807, 504, 906, 903, 907, 702, 904, 805, 902
+#define MAKO_JKSWAP_PICK 703, 803, 706, 503, 802, 806, 901, 804, 502, 807, 504, 906, 903, 907, 702, 904, 805, 902, 905, 908
 #endif
 #ifndef MAKO_SLAB_PICK
 #define MAKO_SLAB_PICK 402

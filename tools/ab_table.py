@@ -27,8 +27,14 @@ RUNS3 = [("r2r_pre", "fec4888 kernels (reference for this group)"),
          ("r2r_superbatch", "slot-batched (dp|pp): R rows of RCAP / K_AB slots per R phase, one primitive quartet per lane (kept)"),
          ("r2r_slab2", "+ (pp|pp) (fs|pp) (fs|dp) (fp|pp) on the slot-batched kernel"),
          ("r2r_slab3", "ket-first classes (dp|ds) (fs|ds) (fp|ps) (fd|ps) (ds|pp) on the slot-batched kernel; (dp|ps) falls to lane-per-ket")]
+# session 3: per-class family re-selection from all-on / all-off runs
+RUNS4 = [("r2s_main", "picks of 82991a3"),
+         ("r2s_tpqx", "every lane-per-ket-eligible light-ket class on the lane-per-ket kernel"),
+         ("r2s_swapall", "every warp-per-quartet class transposed"), ("r2s_swapnone", "no class transposed"),
+         ("r2s_kfnsa", "no ket-first kernel, warp-per-quartet classes transposed"),
+         ("r2s_kfnsn", "no ket-first kernel, nothing transposed")]
 d = {}
-for name, _ in RUNS + RUNS2 + RUNS3:
+for name, _ in RUNS + RUNS2 + RUNS3 + RUNS4:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
     if os.path.exists(p):
         d[name] = json.loads(open(p).read())
@@ -73,3 +79,16 @@ if names3:
     print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names3) + " |")
     for k in classes:
         print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names3) + " |")
+
+names4 = [n for n, _ in RUNS4 if n in d]
+if names4:
+    print("\n## Per-class family re-selection (session 3): (dp|ps) -> lane-per-ket, (ff|dd) (ff|fd) transposed\n")
+    for n, desc in RUNS4:
+        if n in d:
+            print(f"- `{n}`: {desc}")
+    print()
+    print("| class | " + " | ".join(names4) + " |")
+    print("|---|" + "---|" * len(names4))
+    print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names4) + " |")
+    for k in classes:
+        print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names4) + " |")
