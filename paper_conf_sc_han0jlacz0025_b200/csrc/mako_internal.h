@@ -115,7 +115,7 @@ MK_HD constexpr int kgroup(int K) {
 #define MAKO_JK_CAP4 800, 801, 802, 803, 804, 805, 806, 807, 808, 705
 #endif
 #ifndef MAKO_KF_CAP3
-#define MAKO_KF_CAP3 401, 203, 701, 800, 303, 900
+#define MAKO_KF_CAP3 203, 701, 800, 303, 900, 501
 #endif
 constexpr int kKfPick[] = {MAKO_KF_PICK};
 constexpr int kKfSwapPick[] = {MAKO_KFSWAP_PICK};

@@ -33,8 +33,11 @@ RUNS4 = [("r2s_main", "picks of 82991a3"),
          ("r2s_swapall", "every warp-per-quartet class transposed"), ("r2s_swapnone", "no class transposed"),
          ("r2s_kfnsa", "no ket-first kernel, warp-per-quartet classes transposed"),
          ("r2s_kfnsn", "no ket-first kernel, nothing transposed")]
+# session 3: per-class occupancy caps
+RUNS5 = [("r2v_main", "main (tpq kernels compiled with __launch_bounds__(128, 1): the ss-ket classes slower, reverted)"),
+         ("r2v_caps", "(ps|ps) at 5 CTAs/SM; ket-first (dp|ds) (fd|ps) (dd|ps) (fs|ds) at 3 CTAs/SM: only (dd|ps) kept")]
 d = {}
-for name, _ in RUNS + RUNS2 + RUNS3 + RUNS4:
+for name, _ in RUNS + RUNS2 + RUNS3 + RUNS4 + RUNS5:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
     if os.path.exists(p):
         d[name] = json.loads(open(p).read())
@@ -92,3 +95,16 @@ if names4:
     print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names4) + " |")
     for k in classes:
         print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names4) + " |")
+
+names5 = [n for n, _ in RUNS5 if n in d]
+if names5:
+    print("\n## Occupancy caps per class (session 3)\n")
+    for n, desc in RUNS5:
+        if n in d:
+            print(f"- `{n}`: {desc}")
+    print()
+    print("| class | " + " | ".join(names5) + " |")
+    print("|---|" + "---|" * len(names5))
+    print("| **build s** | " + " | ".join("%.3f" % d[n]["s_per_iter"] for n in names5) + " |")
+    for k in classes:
+        print(f"| {k} | " + " | ".join("%.1f" % d[n]["class_ms"][k][0] if k in d[n]["class_ms"] else "" for n in names5) + " |")
