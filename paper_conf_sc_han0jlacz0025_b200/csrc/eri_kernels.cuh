@@ -301,7 +301,7 @@ int jk_blocks_per_sm() {
       if (set_smem_attr<X, Y>((const void*)kf_jk_kernel_ptr<X, Y>(), ks)) return 1;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kf_jk_kernel_ptr<X, Y>(), CTA_THREADS, ks);
     } else if constexpr (use_tpq(X, Y)) {
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, tpq_jk_kernel<X, Y>, CTA_THREADS, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, tpq_jk_kernel_ptr<X, Y>(), CTA_THREADS, 0);
     } else if constexpr (use_slab<X, Y>()) {
       constexpr size_t ss = SlabCfg<X, Y>::SMEM;
       if (set_smem_attr<X, Y>((const void*)slab_jk_kernel<X, Y>, ss)) return 1;
@@ -392,8 +392,8 @@ mako_status launch_jk_xy(const JKArgs& a, void* stream, int* nlaunch) {
       if (a.dsh) tpq_strip_kernel<X, Y, true><<<(int)std::max<long long>(gs, 1), 32 * TPQ_STRIP_WARPS, ss, cs>>>(a);
       else tpq_strip_kernel<X, Y><<<(int)std::max<long long>(gs, 1), 32 * TPQ_STRIP_WARPS, ss, cs>>>(a);
     } else {
-      if (a.dsh) tpq_jk_kernel<X, Y, true><<<grid, CTA_THREADS, 0, cs>>>(a);
-      else tpq_jk_kernel<X, Y><<<grid, CTA_THREADS, 0, cs>>>(a);
+      if (a.dsh) tpq_jk_kernel_ptr<X, Y, true>()<<<grid, CTA_THREADS, 0, cs>>>(a);
+      else tpq_jk_kernel_ptr<X, Y>()<<<grid, CTA_THREADS, 0, cs>>>(a);
     }
   } else if constexpr (use_slab<X, Y>()) {
     if (a.dsh) {

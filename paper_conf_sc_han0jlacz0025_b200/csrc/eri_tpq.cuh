@@ -446,14 +446,37 @@ __device__ __forceinline__ void tpq_task(const JKArgs& a, int P, int r0, int r1,
       }
 }
 
-// Persistent lane-per-ket kernel (JKArgs.KT must be 32).
-#ifdef MAKO_TPQ_MINB
-#define MAKO_TPQ_BOUNDS __launch_bounds__(128, MAKO_TPQ_MINB)
-#else
-#define MAKO_TPQ_BOUNDS __launch_bounds__(128)
+// Persistent lane-per-ket kernel (JKArgs.KT must be 32).  The classes of MAKO_TPQ_CAP3 / MAKO_TPQ_CAP4 are
+// compiled for at least 3 / 4 resident CTAs per SM (register caps 168 / 128; measured per class), the
+// others without a cap.
+#ifndef MAKO_TPQ_CAP3
+#define MAKO_TPQ_CAP3 201, 301, 601  // (pp|ps) (ds|ps) (fs|ps): 2 -> 3 CTAs/SM, 380 -> 375, 407 -> 385, 260 -> 241 ms
 #endif
+#ifndef MAKO_TPQ_CAP4
+#define MAKO_TPQ_CAP4 9999
+#endif
+constexpr int kTpqCap3[] = {MAKO_TPQ_CAP3};
+constexpr int kTpqCap4[] = {MAKO_TPQ_CAP4};
+template <int X, int Y>
+constexpr int tpq_minb() {
+  return in_list(kTpqCap4, X * 100 + Y) ? 4 : (in_list(kTpqCap3, X * 100 + Y) ? 3 : 1);
+}
+template <int X, int Y, bool DW>
+__device__ __forceinline__ void tpq_body(const JKArgs& a);
 template <int X, int Y, bool DW = false>
-__global__ void MAKO_TPQ_BOUNDS tpq_jk_kernel(JKArgs a) {
+__global__ void __launch_bounds__(128) tpq_kernel_free(JKArgs a) { tpq_body<X, Y, DW>(a); }
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(128, 3) tpq_kernel_cap3(JKArgs a) { tpq_body<X, Y, DW>(a); }
+template <int X, int Y, bool DW = false>
+__global__ void __launch_bounds__(128, 4) tpq_kernel_cap4(JKArgs a) { tpq_body<X, Y, DW>(a); }
+template <int X, int Y, bool DW = false>
+constexpr auto tpq_jk_kernel_ptr() {
+  if constexpr (tpq_minb<X, Y>() == 4) return &tpq_kernel_cap4<X, Y, DW>;
+  else if constexpr (tpq_minb<X, Y>() == 3) return &tpq_kernel_cap3<X, Y, DW>;
+  else return &tpq_kernel_free<X, Y, DW>;
+}
+template <int X, int Y, bool DW>
+__device__ __forceinline__ void tpq_body(const JKArgs& a) {
   const int lane = threadIdx.x & 31;
   __shared__ double stage_all[MAKO_TPQ_STAGE ? 4 * tpq_stage_doubles<ClsXY<X, Y>>() : 1];
   double* stage = stage_all + (MAKO_TPQ_STAGE ? (threadIdx.x >> 5) * tpq_stage_doubles<ClsXY<X, Y>>() : 0);

@@ -35,7 +35,10 @@ RUNS4 = [("r2s_main", "picks of 82991a3"),
          ("r2s_kfnsn", "no ket-first kernel, nothing transposed")]
 # session 3: per-class occupancy caps
 RUNS5 = [("r2v_main", "main (tpq kernels compiled with __launch_bounds__(128, 1): the ss-ket classes slower, reverted)"),
-         ("r2v_caps", "(ps|ps) at 5 CTAs/SM; ket-first (dp|ds) (fd|ps) (dd|ps) (fs|ds) at 3 CTAs/SM: only (dd|ps) kept")]
+         ("r2v_caps", "(ps|ps) at 5 CTAs/SM; ket-first (dp|ds) (fd|ps) (dd|ps) (fs|ds) at 3 CTAs/SM: only (dd|ps) kept"),
+         ("r2x_main", "lane-per-ket kernel refactored into free / capped instantiations, no caps"),
+         ("r2x_tpqcap3", "lane-per-ket (pp|ps) (ds|ps) (fs|ps) at 3 CTAs/SM (168 registers, 64-324 B spills): kept"),
+         ("r2x_tpqcap4", "(ds|ps) (fs|ps) at 4 CTAs/SM, (pp|ps) at 3: slower")]
 d = {}
 for name, _ in RUNS + RUNS2 + RUNS3 + RUNS4 + RUNS5:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
