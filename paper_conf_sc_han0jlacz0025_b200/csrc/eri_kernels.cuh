@@ -69,7 +69,8 @@ __host__ __device__ constexpr size_t cta_smem_bytes() {
   return (size_t)C::HTAB_BYTES + C::RTAB_BYTES + sizeof(double) * (size_t)jk_warps<C>() * C::WARP_DBL;
 }
 
-// occupancy cap (4 CTAs/SM, <= 128 registers) measured faster for the fd-bra classes and (fp|dd) only
+// occupancy cap (4 CTAs/SM, <= 128 registers) measured faster for the fd-bra classes, (fp|dd), and (round 2,
+// codes of the evaluated orientation) the transposed (fd|dp) (ff|pp) (ff|fs); (fd|fd) runs uncapped
 template <int X, int Y>
 constexpr int jk_minb() {
   return in_list(kJkCap4, X * 100 + Y) ? 4 : 1;

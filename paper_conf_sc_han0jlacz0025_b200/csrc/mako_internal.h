@@ -112,7 +112,7 @@ MK_HD constexpr int kgroup(int K) {
 #define MAKO_SLAB_PICK 402
 #endif
 #ifndef MAKO_JK_CAP4
-#define MAKO_JK_CAP4 800, 801, 802, 803, 804, 805, 806, 807, 808, 705
+#define MAKO_JK_CAP4 800, 801, 802, 803, 804, 805, 806, 807, 705, 408, 209, 609
 #endif
 #ifndef MAKO_KF_CAP3
 #define MAKO_KF_CAP3 203, 701, 800, 303, 900, 501

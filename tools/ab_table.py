@@ -38,7 +38,10 @@ RUNS5 = [("r2v_main", "main (tpq kernels compiled with __launch_bounds__(128, 1)
          ("r2v_caps", "(ps|ps) at 5 CTAs/SM; ket-first (dp|ds) (fd|ps) (dd|ps) (fs|ds) at 3 CTAs/SM: only (dd|ps) kept"),
          ("r2x_main", "lane-per-ket kernel refactored into free / capped instantiations, no caps"),
          ("r2x_tpqcap3", "lane-per-ket (pp|ps) (ds|ps) (fs|ps) at 3 CTAs/SM (168 registers, 64-324 B spills): kept"),
-         ("r2x_tpqcap4", "(ds|ps) (fs|ps) at 4 CTAs/SM, (pp|ps) at 3: slower")]
+         ("r2x_tpqcap4", "(ds|ps) (fs|ps) at 4 CTAs/SM, (pp|ps) at 3: slower"),
+         ("r2y_main", "main with the lane-per-ket caps (ef7f4a2)"),
+         ("r2z_jkcap", "every warp-per-quartet class at 4 CTAs/SM: kept for (fd|dp) (ff|pp) (ff|fs)"),
+         ("r2z_jknocap", "no warp-per-quartet class capped: kept for (fd|fd)")]
 d = {}
 for name, _ in RUNS + RUNS2 + RUNS3 + RUNS4 + RUNS5:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
