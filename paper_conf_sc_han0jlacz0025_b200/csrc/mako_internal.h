@@ -124,7 +124,7 @@ constexpr int kJkSwapPick[] = {MAKO_JKSWAP_PICK};
 // warp-per-quartet classes (codes bucket(la,lb) * 100 + bucket(lc,ld) of the evaluated orientation)
 // whose contracted quartets take the batched lane-per-quartet R path (eri_core.cuh quartet_block_rb)
 #ifndef MAKO_RBATCH_PICK
-#define MAKO_RBATCH_PICK 207, 205, 602, 404, 202
+#define MAKO_RBATCH_PICK 207, 205, 602, 404, 202, 307
 #endif
 constexpr int kRBatchPick[] = {MAKO_RBATCH_PICK};
 // warp-per-quartet classes (same codes) whose GEMM2 B operands are read from the row-major E~ rather

@@ -41,7 +41,12 @@ RUNS5 = [("r2v_main", "main (tpq kernels compiled with __launch_bounds__(128, 1)
          ("r2x_tpqcap4", "(ds|ps) (fs|ps) at 4 CTAs/SM, (pp|ps) at 3: slower"),
          ("r2y_main", "main with the lane-per-ket caps (ef7f4a2)"),
          ("r2z_jkcap", "every warp-per-quartet class at 4 CTAs/SM: kept for (fd|dp) (ff|pp) (ff|fs)"),
-         ("r2z_jknocap", "no warp-per-quartet class capped: kept for (fd|fd)")]
+         ("r2z_jknocap", "no warp-per-quartet class capped: kept for (fd|fd)"),
+         ("r2f2_main", "main with the re-selected caps (015c565)"),
+         ("r2sw_rball", "batched lane-per-quartet R for every warp-per-quartet class with L <= 6: kept for (fp|ds)"),
+         ("r2sw_rbnone", "batched R for none"),
+         ("r2sw_fball", "GEMM2 B operands from the fragment-order copy for every class"),
+         ("r2sw_fbnone", "... for none (row-major E~)")]
 d = {}
 for name, _ in RUNS + RUNS2 + RUNS3 + RUNS4 + RUNS5:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
