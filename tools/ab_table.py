@@ -46,7 +46,9 @@ RUNS5 = [("r2v_main", "main (tpq kernels compiled with __launch_bounds__(128, 1)
          ("r2sw_rball", "batched lane-per-quartet R for every warp-per-quartet class with L <= 6: kept for (fp|ds)"),
          ("r2sw_rbnone", "batched R for none"),
          ("r2sw_fball", "GEMM2 B operands from the fragment-order copy for every class"),
-         ("r2sw_fbnone", "... for none (row-major E~)")]
+         ("r2sw_fbnone", "... for none (row-major E~)"),
+         ("r2f3_main", "final kernels (076314d)"),
+         ("r2kc_kfnocap", "no 3-CTA register cap on any ket-first class: every cap of the list still pays ((ds|pp) 551 -> 637 ms without)")]
 d = {}
 for name, _ in RUNS + RUNS2 + RUNS3 + RUNS4 + RUNS5:
     p = os.path.join(ROOT, "profiles", "ab_r02", name + ".jsonl")
